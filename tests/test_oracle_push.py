@@ -1,0 +1,291 @@
+"""Pins for the oracle's push / move / deposit (VPIC reading).
+
+Expected values come from physics and geometry, not from the oracle:
+* uniform E, B = 0: u_n = u_0 + 2 n qdt_2mc E, bit-exact for dyadic inputs;
+  position advances by u c dt / (gamma dx) per step (relativistic velocity);
+* uniform B: |u| conserved (the Boris rotation is a rotation); the rotation
+  angle per step equals the exact cyclotron angle 2 phi = 2 qdt_2mc |B| / gamma
+  up to the O(phi^7) remainder of the 5th-order tan series that the
+  tan-corrected Boris uses (reading R11); positive charges turn clockwise
+  about B; the orbit is a regular polygon: chord L = |u| c dt / gamma and
+  circumradius R = L / (2 sin(theta/2));
+* E x B: the guiding centre drifts at E x B / B^2;
+* move_p: offsets stay in [-1,1]; the global displacement telescopes to the
+  requested one; reflect mirrors; absorb / remote report the exit face;
+* charge conservation: 4 (R_new - R_old) + div J = 0 at every node
+  (Delta rho + Delta t div J = 0, the discrete continuity invariant);
+* deposit totals: sum of all jx partials = 4 sum q disp_x.
+"""
+import math
+
+import numpy as np
+import pytest
+
+from paper_conf_sc_tanlta25_b200 import inputs
+
+PD = inputs.PARTICLE_DTYPE
+
+
+def grid(n=4, dt=0.5, pbc=(0,) * 6, nbr=(0,) * 6):
+    return inputs.GridSpec(n, n, n, dt=dt, pbc=tuple(pbc), nbr_rank=tuple(nbr))
+
+
+def uniform_fields(g, E=(0, 0, 0), B=(0, 0, 0)):
+    f = np.zeros((g.nv, 8), np.float32)
+    f[:, 0:3] = np.array(E, np.float32)
+    f[:, 4:7] = np.array(B, np.float32)
+    return f
+
+
+def one_particle(g, cell=(2, 2, 2), d=(0, 0, 0), u=(0, 0, 0), w=1.0):
+    p = np.zeros(1, PD)
+    p["i"] = g.voxel(*cell)
+    p["dx"], p["dy"], p["dz"] = d
+    p["ux"], p["uy"], p["uz"] = u
+    p["w"] = w
+    return p
+
+
+def global_pos(g, p):
+    """Physical position in cell units: voxel (x,y,z) spans [x, x+1]."""
+    x, y, z = g.coords(p["i"])
+    return np.stack([x + (1 + p["dx"].astype(np.float64)) / 2,
+                     y + (1 + p["dy"].astype(np.float64)) / 2,
+                     z + (1 + p["dz"].astype(np.float64)) / 2], -1)
+
+
+def unwrap_step(prev, cur, n):
+    d = cur - prev
+    return d - n * np.round(d / n)
+
+
+def run(orc, g, p, fields, q, m, steps, track=False):
+    interp = orc.load_interpolator(g, fields)
+    acc = np.zeros((g.nv, 12), np.float32)
+    us, xs = [], []
+    pos = global_pos(g, p)
+    disp = np.zeros_like(pos)
+    for _ in range(steps):
+        acc[:] = 0
+        mv = orc.advance_p(g, q, m, p, interp, acc)
+        assert mv.size == 0
+        new = global_pos(g, p)
+        disp += unwrap_step(pos, new, np.array([g.nx, g.ny, g.nz]))
+        pos = new
+        if track:
+            us.append(np.array([p["ux"][0], p["uy"][0], p["uz"][0]], np.float64))
+            xs.append(disp[0].copy())
+    return np.array(us), np.array(xs)
+
+
+def test_uniform_E_bit_exact(orc):
+    """TV1: qdt_2mc = 1/4, E = (2^-8, -2^-9, 2^-7)."""
+    g = grid(dt=0.5)
+    E = (2.0**-8, -(2.0**-9), 2.0**-7)
+    p = one_particle(g)
+    us, xs = run(orc, g, p, uniform_fields(g, E=E), 1.0, 1.0, 300, track=True)
+    n = np.arange(1, 301)[:, None]
+    expect = n * 2 * 0.25 * np.array(E)
+    assert np.array_equal(us, expect)  # bit-exact
+    # position: sum_n u_n c dt / gamma_n (cells), in double
+    gam = np.sqrt(1 + (expect**2).sum(1))[:, None]
+    xexp = np.cumsum(expect * 0.5 / gam, 0)
+    assert np.abs(xs - xexp).max() < 2e-5
+    assert abs(xs[-1, 0]) > 4  # crossed the periodic box more than once
+
+
+def test_gyration(orc):
+    """TV2: qdt_2mc = 0.3, cB = (0,0,1.3), u0 = (0.4,0,0), E = 0."""
+    g = grid(dt=0.6)
+    p = one_particle(g, u=(0.4, 0.0, 0.0))
+    us, xs = run(orc, g, p, uniform_fields(g, B=(0, 0, 1.3)), 1.0, 1.0, 2000, track=True)
+    umag = np.linalg.norm(us, axis=1)
+    assert np.abs(umag - 0.4).max() < 4e-6          # energy conserved
+    assert np.all(us[:, 2] == 0)
+    ang = np.arctan2(us[:, 1], us[:, 0])
+    dth = np.diff(np.concatenate([[0.0], ang]))
+    dth = (dth + np.pi) % (2 * np.pi) - np.pi
+    assert np.all(dth < 0)                          # q > 0 turns clockwise about +z
+    gamma = math.sqrt(1 + 0.16)
+    phi = 0.3 * 1.3 / gamma
+    theta = -dth.mean()
+    remainder = 2 * (17.0 / 315.0) * phi**7
+    assert abs(theta - 2 * phi) < 1.5 * remainder + 1e-6
+    assert abs(theta - 2 * phi) > 0.3 * remainder   # the tan correction is truncated, not exact
+    # regular polygon: chord and circumradius
+    L = 0.4 * 0.6 / gamma
+    chords = np.linalg.norm(np.diff(xs[:, :2], axis=0), axis=1)
+    assert np.abs(chords - L).max() < 2e-6
+    a = xs[:-2, :2]; b = xs[1:-1, :2]; c = xs[2:, :2]
+    la = np.linalg.norm(b - c, axis=1); lb = np.linalg.norm(a - c, axis=1); lc = np.linalg.norm(a - b, axis=1)
+    area = 0.5 * np.abs((b - a)[:, 0] * (c - a)[:, 1] - (b - a)[:, 1] * (c - a)[:, 0])
+    R = np.median(la * lb * lc / (4 * area))
+    assert abs(R - L / (2 * math.sin(theta / 2))) / R < 2e-4
+
+
+def test_ExB_drift(orc):
+    """Small phi: the particle started at the drift speed keeps E x B / B^2."""
+    g = grid(dt=0.05)
+    vd = 0.01
+    p = one_particle(g, u=(vd / math.sqrt(1 - vd * vd), 0, 0))
+    steps = 4000
+    us, xs = run(orc, g, p, uniform_fields(g, E=(0, vd, 0), B=(0, 0, 1.0)), 1.0, 1.0, steps, track=True)
+    v = xs[-1] / (steps * 0.05)
+    assert abs(v[0] - vd) / vd < 2e-3
+    assert abs(v[1]) < 1e-5 and v[2] == 0
+
+
+def test_ExB_drift_negative_charge(orc):
+    g = grid(dt=0.05)
+    vd = 0.01
+    p = one_particle(g, u=(vd / math.sqrt(1 - vd * vd), 0, 0))
+    steps = 4000
+    _, xs = run(orc, g, p, uniform_fields(g, E=(0, vd, 0), B=(0, 0, 1.0)), -1.0, 1.0, steps, track=True)
+    v = xs[-1] / (steps * 0.05)
+    assert abs(v[0] - vd) / vd < 2e-3   # E x B drift is charge independent
+
+
+def _random_movers(g, n, seed, scale=0.99):
+    rng = np.random.default_rng(seed)
+    p = inputs.random_particles(g, n, seed)
+    disp = (rng.random((n, 3)) * 2 - 1) * scale
+    return p, disp.astype(np.float32)
+
+
+def test_move_p_geometry_periodic(orc):
+    g = grid(n=3)
+    p, disp = _random_movers(g, 3000, 5)
+    # put some particles exactly on faces and give some zero displacement
+    p["dx"][:100] = 1.0
+    p["dy"][100:200] = -1.0
+    disp[200:300, 1] = 0.0
+    acc = np.zeros((g.nv, 12), np.float32)
+    pos0 = global_pos(g, p)
+    for k in range(p.size):
+        pk = p[k:k + 1].copy()
+        mv = _mover(disp[k])
+        assert orc.move_p(g, pk, mv, acc, 1.0) == 0
+        assert mv["dispx"][0] == 0 or abs(mv["dispx"][0]) < 1e-6
+        p[k] = pk[0]
+    assert np.all(np.abs(p["dx"]) <= 1) and np.all(np.abs(p["dy"]) <= 1) and np.all(np.abs(p["dz"]) <= 1)
+    x, y, z = g.coords(p["i"])
+    assert np.all((x >= 1) & (x <= 3) & (y >= 1) & (y <= 3) & (z >= 1) & (z <= 3))
+    moved = unwrap_step(pos0, global_pos(g, p), np.array([3, 3, 3]))
+    assert np.abs(moved - disp.astype(np.float64)).max() < 2e-6
+
+
+def _mover(d):
+    mv = np.zeros(1, np.dtype([("dispx", "<f4"), ("dispy", "<f4"), ("dispz", "<f4"), ("idx", "<i4")]))
+    mv["dispx"], mv["dispy"], mv["dispz"] = d
+    return mv
+
+
+def test_move_p_reflect_absorb_remote(orc):
+    g = grid(n=4, pbc=(0, 0, 1, 0, 0, 2), nbr=(0, 0, 0, 0, 1, 0))
+    acc = np.zeros((g.nv, 12), np.float32)
+    # reflect at -z: z=1 cell, offset -0.5, moving -z by 0.5 cells (disp 0.5 offset units -> 1.0)
+    p = one_particle(g, cell=(2, 2, 1), d=(0, 0, -0.5), u=(0, 0, -0.3))
+    X0 = global_pos(g, p)[0]
+    assert orc.move_p(g, p, _mover((0.1, 0.0, -0.5)), acc, 1.0) == 0
+    X1 = global_pos(g, p)[0]
+    assert p["uz"][0] == np.float32(0.3)
+    # unreflected z would be X0 - 0.5 = 0.75 - 0.5 = 0.25 -> mirrored about z=1 -> 1.75
+    assert abs(X1[2] - (2 * 1.0 - (X0[2] - 0.5))) < 1e-6
+    assert abs(X1[0] - (X0[0] + 0.1)) < 1e-6
+    # absorb at +z
+    p = one_particle(g, cell=(3, 1, 4), d=(0.2, 0, 0.5), u=(0, 0, 0.3))
+    mv = _mover((0.0, 0.0, 0.5))
+    assert orc.move_p(g, p, mv, acc, 1.0) == 1
+    assert p["i"][0] == 8 * g.voxel(3, 1, 4) + 5 and p["dz"][0] == 1.0
+    assert abs(mv["dispz"][0] - 0.25) < 1e-7
+    # remote at +y (nbr_rank[+y] = 1 != rank 0)
+    p = one_particle(g, cell=(1, 4, 2), d=(0, 0.9, 0), u=(0, 0.3, 0))
+    mv = _mover((0.0, 0.2, 0.0))
+    assert orc.move_p(g, p, mv, acc, 1.0) == 1
+    assert p["i"][0] == 8 * g.voxel(1, 4, 2) + 4 and p["dy"][0] == 1.0
+    assert abs(mv["dispy"][0] - 0.15) < 1e-7
+
+
+def _continuity(orc, g, n, seed, fields_amp, q=0.7, perturb=0.0):
+    rng = np.random.default_rng(seed)
+    p = inputs.random_particles(g, n, seed, u_scale=0.8)
+    fields = (rng.random((g.nv, 8)) * 2 - 1).astype(np.float32) * np.float32(fields_amp)
+    interp = orc.load_interpolator(g, fields)
+    acc = np.zeros((g.nv, 12), np.float32)
+    rho0 = orc.accumulate_rho(g, p, q)
+    orc.advance_p(g, q, 1.0, p, interp, acc)
+    rho1 = orc.accumulate_rho(g, p, q)
+    if perturb:
+        acc = acc * np.float32(1 + perturb)
+    J = orc.unload_raw(g, acc)
+    n3 = (g.nx, g.ny, g.nz)
+    S = (g.nx + 2, g.ny + 2, g.nz + 2)
+    Jg = J[:, :3].reshape(S[2], S[1], S[0], 3).transpose(2, 1, 0, 3).copy()  # [x,y,z,c]
+    R = (rho1 - rho0).reshape(S[2], S[1], S[0]).transpose(2, 1, 0)
+    per = [g.pbc[a] == 0 for a in range(3)]
+    for a in range(3):  # fold periodic planes n+1 -> 1
+        if per[a]:
+            sl_hi = [slice(None)] * 3; sl_hi[a] = n3[a] + 1
+            sl_lo = [slice(None)] * 3; sl_lo[a] = 1
+            Jg[tuple(sl_lo)] += Jg[tuple(sl_hi)]
+            Jg[tuple(sl_hi)] = 0
+            R[tuple(sl_lo)] += R[tuple(sl_hi)]
+            R[tuple(sl_hi)] = 0
+    res = 4 * R
+    for a in range(3):
+        Ja = Jg[..., a]
+        if per[a]:
+            # J(n) - J(n - e) with periodic wrap over interior planes 1..n
+            core = np.take(Ja, np.arange(1, n3[a] + 1), axis=a)
+            div = core - np.roll(core, 1, axis=a)
+            pad = np.zeros_like(Ja)
+            put = [slice(None)] * 3; put[a] = slice(1, n3[a] + 1)
+            pad[tuple(put)] = div
+            res = res + pad
+        else:
+            shifted = np.zeros_like(Ja)
+            s_dst = [slice(None)] * 3; s_dst[a] = slice(1, None)
+            s_src = [slice(None)] * 3; s_src[a] = slice(0, -1)
+            shifted[tuple(s_dst)] = Ja[tuple(s_src)]
+            res = res + (Ja - shifted)
+    return np.abs(res).max(), np.abs(4 * R).max(), p, acc
+
+
+@pytest.mark.parametrize("seed", [0, 1])
+def test_continuity_periodic(orc, seed):
+    g = grid(n=4, dt=0.5)
+    resid, scale, _, _ = _continuity(orc, g, 2000, seed, 0.05)
+    assert scale > 1.0
+    assert resid < 2e-5 * max(1.0, scale), (resid, scale)
+
+
+def test_continuity_reflect_z(orc):
+    g = grid(n=4, dt=0.5, pbc=(0, 0, 1, 0, 0, 1))
+    resid, scale, p, _ = _continuity(orc, g, 2000, 7, 0.05)
+    assert scale > 1.0
+    assert resid < 2e-5 * max(1.0, scale)
+
+
+def test_continuity_detects_wrong_current(orc):
+    """Sanity of the pin itself: a 1% current error is caught."""
+    g = grid(n=4, dt=0.5)
+    resid, scale, _, _ = _continuity(orc, g, 2000, 3, 0.0, perturb=0.01)
+    assert resid > 1e-3 * scale
+
+
+def test_deposit_totals(orc):
+    g = grid(n=5, dt=0.5)
+    q = -0.7
+    p = inputs.random_particles(g, 3000, 11, u_scale=0.9)
+    interp = np.zeros((g.nv, 20), np.float32)
+    acc = np.zeros((g.nv, 12), np.float32)
+    acc_abs = np.zeros((g.nv, 12), np.float64)
+    u = np.stack([p["ux"], p["uy"], p["uz"]], 1).astype(np.float64)
+    gam = np.sqrt(1 + (u**2).sum(1))
+    disp = u * 0.5 / gam[:, None]          # half displacement, cdt_dx = 0.5
+    qw = q * p["w"].astype(np.float64)
+    orc.advance_p(g, q, 1.0, p, interp, acc, acc_abs)
+    for a in range(3):
+        tot = acc[:, 4 * a:4 * a + 4].astype(np.float64).sum()
+        exp = 4 * (qw * disp[:, a]).sum()
+        assert abs(tot - exp) < 1e-5 * acc_abs[:, 4 * a:4 * a + 4].sum()

@@ -1,0 +1,373 @@
+#!/usr/bin/env python
+"""Benchmark of the VPIC particle hot path on B200 (BASELINE.json metric:
+particle pushes/sec (advance_p + sort) per GPU and at N GPUs; % of HBM roofline).
+
+One bench step = one sort period of the workload: vpic_sort_particles (per
+species) followed by S = sort_every PIC steps of load_interpolator ->
+clear_accumulator -> advance_p (per species) [-> migrate] ->
+unload_accumulator, all through the C-ABI on device-resident inputs
+(BASELINE.json configs[1]: uniform 128^3, 128 ppc/species, sort every 20).
+value = pushes (particles x PIC steps, all ranks) / max-over-ranks device time.
+
+    python bench.py [--gpus N --steps K --warmup W]           # our arm
+    python bench.py --impl reference [...]                    # the oracle on host cores
+N > 1: launch with torch.distributed.run (one rank per GPU, NCCL); the box is
+weak-scaled (a 128^3 block per GPU, BASELINE.json configs[3]).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+FALLBACK_HBM_GBS = 6650.0
+METRIC = "particle pushes/sec (advance_p+sort)"
+UNIT = "pushes/s"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", type=int, default=1)
+    ap.add_argument("--order", default="standard", choices=["standard", "strided", "tiled_strided", "none"])
+    ap.add_argument("--shuffle", action="store_true", help="random initial order (paper's 'random')")
+    ap.add_argument("--sort-every", type=int, default=0)
+    ap.add_argument("--math", default="fast", choices=["fast", "ieee"])
+    ap.add_argument("--deposit", default="auto", choices=["auto", "lane", "warp"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--profile", action="store_true", help="short run for ncu (no e2e/cpu legs)")
+    return ap.parse_args()
+
+
+ORDERS = {"standard": 0, "strided": 1, "tiled_strided": 2, "none": 3}
+
+
+# ------------------------------------------------------------ helpers --
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons during the timed region."""
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+             "clocks_event_reasons.sw_power_cap")
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={q}", "--format=csv,noheader,nounits",
+                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thread = threading.Thread(target=self._read, daemon=True)
+            self.thread.start()
+        except FileNotFoundError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) == 7:
+                self.rows.append(parts)
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[k] for r in self.rows for k in range(4) if r[3 + k].lower() == "active"})
+        load = [s for s in sm]
+        return {"sm_mhz": statistics.median(load) if load else None,
+                "sm_max_mhz": max(mx) if mx else None, "reasons": reasons, "samples": len(self.rows)}
+
+
+def hbm_peak():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(path) as f:
+            return float(json.load(f)["hbm_gbs"]), "measured"
+    except Exception:
+        return FALLBACK_HBM_GBS, "fallback"
+
+
+def committed_traffic(kernel_key: str, workload: str):
+    """dram bytes per launch of the dominant kernel from the committed ncu
+    --set full summary (profiles/traffic.json), if it matches this workload."""
+    path = os.path.join(ROOT, "profiles", "traffic.json")
+    try:
+        with open(path) as f:
+            t = json.load(f)
+        e = t.get(kernel_key, {})
+        if e.get("workload") == workload:
+            return e.get("dram_bytes_per_launch"), e
+    except Exception:
+        pass
+    return None, None
+
+
+# --------------------------------------------------------- CPU / oracle --
+def oracle_sample_workload():
+    """The reference arm's bounded sample: the same plasma recipe (species,
+    ppc, u_th, fields, sort period) on a 32x32x16 box."""
+    from paper_conf_sc_tanlta25_b200 import inputs
+    from dataclasses import replace
+    wl = inputs.config(1)
+    return replace(wl, grid=inputs.GridSpec(32, 32, 16), name=wl.name + "@32x32x16")
+
+
+def run_oracle_steps(wl, n_steps, sort_every, order):
+    import oracle
+    from paper_conf_sc_tanlta25_b200 import inputs
+    oracle.build()
+    g = wl.grid
+    parts = inputs.make_species_particles(wl)
+    fields = inputs.make_fields(g, wl.field_amp)
+    acc = np.zeros((g.nv, 12), np.float32)
+    times = []
+    pushes = 0
+    for step in range(n_steps):
+        t0 = time.perf_counter()
+        for k in range(sort_every):
+            if k == 0 and order != 3:
+                parts = [oracle.sort_particles(g, p, order, 3 * 148 * 128)[0] for p in parts]
+            interp = oracle.load_interpolator(g, fields)
+            acc[:] = 0
+            for sp, p in zip(wl.species, parts):
+                oracle.advance_p(g, sp.q, sp.m, p, interp, acc)
+                pushes += p.size
+            oracle.unload_accumulator(g, acc)
+        times.append(time.perf_counter() - t0)
+    return times, sum(p.size for p in parts) * sort_every
+
+
+def reference_arm(args, rank, world):
+    if rank != 0:
+        return
+    wl = oracle_sample_workload()
+    S = args.sort_every or wl.sort_every
+    order = ORDERS[args.order]
+    _ = run_oracle_steps(wl, max(args.warmup, 0) and 1, S, order)  # untimed warm-up (1 step)
+    times, per_step = run_oracle_steps(wl, args.steps, S, order)
+    total = sum(times)
+    value = per_step * args.steps / total
+    out = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * total / args.steps,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+        "data": "synthetic",
+        "config": {"workload": wl.name, "order": args.order, "sort_every": S,
+                   "particles": per_step // S},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
+                         "sample": f"serial C++ oracle (oracle/), {wl.name}: {per_step // S} particles, "
+                                   f"sort + {S} PIC steps per step"},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(out), flush=True)
+
+
+def cpu_baseline(args):
+    wl = oracle_sample_workload()
+    S = args.sort_every or wl.sort_every
+    times, per_step = run_oracle_steps(wl, 1, S, ORDERS[args.order])
+    return {"value": per_step / times[0], "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"serial C++ oracle on {wl.name} ({per_step // S} particles): one sort + {S} "
+                      f"PIC steps, {times[0]:.1f} s on 1 host core"}
+
+
+# ---------------------------------------------------------------- ours --
+def our_arm(args, rank, world):
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_tanlta25_b200 import inputs, vpic
+    from paper_conf_sc_tanlta25_b200.pic import HotPath
+
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    wl = inputs.config(3 if world > 1 else args.config)
+    S = args.sort_every or wl.sort_every
+    order = ORDERS[args.order]
+    g = inputs.decompose(wl.grid, world, rank) if world > 1 else wl.grid
+    from dataclasses import replace
+    wl = replace(wl, grid=g)
+    uid = None
+    if world > 1:
+        obj = [vpic.vpic_get_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        uid = obj[0]
+    seed = inputs.MASTER_SEED + 1 + rank
+    parts = inputs.make_species_particles(wl, seed)
+    if args.shuffle:
+        parts = [inputs.shuffle(p, seed + 17 + k) for k, p in enumerate(parts)]
+    fields = inputs.make_fields(g, wl.field_amp, seed)
+    math_mode = vpic.MATH_IEEE if args.math == "ieee" else vpic.MATH_FAST
+    dep = {"auto": 0, "lane": 1, "warp": 2}[args.deposit]
+    cap = 1.0 if world == 1 else 1.05
+    hp = HotPath(wl, parts, fields, order=order, math=math_mode, deposit=dep, rank=rank,
+                 nranks=world, uid=uid, capacity_factor=cap, device=local)
+    n_local = hp.n_particles
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    # ---- warm-up
+    for _ in range(args.warmup):
+        hp.cycle(S)
+    torch.cuda.synchronize()
+    barrier()
+
+    # ---- timed region (device-resident inputs; 17 GB of particles >> 126 MB L2)
+    stream = torch.cuda.current_stream()
+    hp.adv_events = []
+    hp.record_advance = True
+    launches0 = vpic.vpic_kernel_launches()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    pushes_local = 0
+    with ClockSampler(local) as clk:
+        torch.cuda.synchronize()
+        barrier()
+        e0.record(stream)
+        for _ in range(args.steps):
+            hp.cycle(S)
+            pushes_local += S * hp.n_particles
+        e1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+    launches = vpic.vpic_kernel_launches() - launches0
+    hp.record_advance = False
+    ms = e0.elapsed_time(e1)
+    adv = [(a.elapsed_time(b), n) for a, b, n in hp.adv_events]
+    adv_ms = sum(t for t, _ in adv) / len(adv)
+    adv_np = sum(n for _, n in adv) / len(adv)
+    t = torch.tensor([ms, float(pushes_local), float(n_local)], dtype=torch.float64, device=dev)
+    if world > 1:
+        tmax = t.clone()
+        dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
+        tsum = t.clone()
+        dist.all_reduce(tsum, op=dist.ReduceOp.SUM)
+        ms_max, pushes, ntot = float(tmax[0]), float(tsum[1]), float(tsum[2])
+    else:
+        ms_max, pushes, ntot = ms, float(pushes_local), float(n_local)
+    value = pushes / (ms_max / 1e3)
+
+    # ---- e2e: host (pinned) -> device inputs and device -> host results inside the timed region
+    e2e = None
+    if not args.no_e2e and not args.profile:
+        host_in = [torch.from_numpy(np.ascontiguousarray(p).view(np.float32).reshape(-1, 8)).pin_memory()
+                   for p in parts]
+        host_out = [torch.empty(tuple(h.shape), dtype=torch.float32, pin_memory=True) for h in host_in]
+        f_host = torch.from_numpy(fields).pin_memory()
+        jf_host = torch.empty(tuple(hp.jf.shape), dtype=torch.float32, pin_memory=True)
+        h2d = sum(h.numel() * 4 for h in host_in) + f_host.numel() * 4
+        d2h = sum(h.numel() * 4 for h in host_out) + jf_host.numel() * 4
+        torch.cuda.synchronize()
+        barrier()
+        a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a0.record(stream)
+        e2e_pushes = 0
+        for _ in range(args.steps):
+            for s, h in zip(hp.species, host_in):
+                s.p[:h.shape[0]].copy_(h, non_blocking=True)
+                s.np = h.shape[0]
+            hp.fields.copy_(f_host, non_blocking=True)
+            hp.cycle(S)
+            e2e_pushes += S * hp.n_particles
+            for s, h in zip(hp.species, host_out):
+                n = min(s.np, h.shape[0])
+                h[:n].copy_(s.p[:n], non_blocking=True)
+            jf_host.copy_(hp.jf, non_blocking=True)
+        a1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+        ems = a0.elapsed_time(a1)
+        et = torch.tensor([ems, float(e2e_pushes)], dtype=torch.float64, device=dev)
+        if world > 1:
+            em = et.clone(); dist.all_reduce(em, op=dist.ReduceOp.MAX)
+            es = et.clone(); dist.all_reduce(es, op=dist.ReduceOp.SUM)
+            ems, e2e_pushes = float(em[0]), float(es[1])
+        e2e = {"value": e2e_pushes / (ems / 1e3), "unit": UNIT, "h2d_bytes_per_step": h2d,
+               "d2h_bytes_per_step": d2h}
+
+    if rank != 0:
+        return
+    # ---- roofline of the dominant kernel (k_advance: one launch = one species)
+    peak, peak_kind = hbm_peak()
+    ncell = g.nx * g.ny * g.nz
+    alg_bytes = 64.0 * adv_np + (80.0 + 48.0) * ncell
+    achieved = alg_bytes / (adv_ms / 1e3) / 1e9
+    traffic, tinfo = committed_traffic("k_advance", wl.name)
+    adv_share = sum(t for t, _ in adv) / ms
+    clocks = clk.summary()
+    out = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+        "data": "synthetic (seeded Philox; uniform thermal e/ion plasma, quiet start)",
+        "config": {"workload": wl.name, "cells_per_gpu": [g.nx, g.ny, g.nz], "ppc_per_species": wl.ppc,
+                   "species": len(wl.species), "particles": int(ntot), "sort_every": S,
+                   "order": args.order, "shuffled": bool(args.shuffle), "math": args.math,
+                   "deposit": args.deposit, "parallelism": f"domain{world}",
+                   "l2": "no flush: inputs (17 GB of particles per GPU) >> 126 MB L2"},
+        "per_gpu": value / world,
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
+                     "kernel": "k_advance (advance_p, one species per launch)",
+                     "alg_bytes_per_launch": alg_bytes, "avg_launch_ms": adv_ms,
+                     "share_of_step": adv_share, "frac_of_8TBs": achieved / 8000.0},
+        "clocks": clocks,
+        "gpu_launches": launches,
+        "e2e": e2e,
+    }
+    if not args.no_cpu_baseline and not args.profile and world == 1:
+        out["cpu_baseline"] = cpu_baseline(args)
+    print(json.dumps(out), flush=True)
+
+
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if args.impl == "reference":
+        reference_arm(args, rank, world)
+        return
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(int(os.environ.get("LOCAL_RANK", "0")))
+        dist.init_process_group("nccl")
+    try:
+        our_arm(args, rank, world)
+    finally:
+        if world > 1:
+            import torch.distributed as dist
+            dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

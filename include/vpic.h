@@ -1,0 +1,201 @@
+/*
+ * vpic.h -- C ABI of libvpic.so, the B200-native (sm_100a) VPIC particle hot
+ * path of Tan, Luedtke, Taufer & Albright, "Bridging Performance Portability
+ * and Scalability for Plasma Simulations on Heterogeneous Systems", SC
+ * Workshops '25 ("P:L" below = line L of that paper's text, PAPER.md).
+ *
+ * Conventions (all calls):
+ *  - Every array argument is CALLER-OWNED DEVICE memory (e.g. a PyTorch CUDA
+ *    tensor's data_ptr), 16-byte aligned unless stated.  The library never
+ *    frees, retains or reallocates a caller pointer after the call returns.
+ *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default
+ *    stream).  Every call only ENQUEUES work on `stream` and returns without
+ *    synchronising, except vpic_migrate_particles (documented below).
+ *  - Return value: VPIC_OK (0) or a negative vpic_status.  Arguments are
+ *    validated on the host before anything is enqueued; on error nothing is
+ *    enqueued.  No call aborts the process and no C++ exception crosses it.
+ *  - Layouts (all little-endian, no padding beyond what is written):
+ *      voxel index   v = x + (nx+2)*(y + (ny+2)*z), interior x in 1..nx etc.,
+ *                    nv = (nx+2)(ny+2)(nz+2) voxels including one ghost layer;
+ *      particle      vpic_particle_t, 32 B (AoS);
+ *      fields[nv][8] float: ex,ey,ez,0, cbx,cby,cbz,0 (Yee: ex on the x-edge
+ *                    from node (x,y,z) to (x+1,y,z), cbx on the -x face);
+ *      interp[nv][20] float: ex,dexdy,dexdz,d2exdydz, ey,deydz,deydx,
+ *                    d2eydzdx, ez,dezdx,dezdy,d2ezdxdy, cbx,dcbxdx,
+ *                    cby,dcbydy, cbz,dcbzdz, 0,0  (80 B = 5 x float4);
+ *      acc[nv][12]   float: jx[4], jy[4], jz[4] quadrant partials
+ *                    (48 B = 3 x float4); jx quadrants (-y-z),(+y-z),(-y+z),(+y+z),
+ *                    jy cyclic over (z,x), jz over (x,y);
+ *      jf[nv][4]     float: jfx, jfy, jfz, 0 on the Yee edges.
+ *    The push, move, deposit, interpolation and unload formulas are the VPIC
+ *    algorithms the paper relies on (ref. [3]); DESIGN.md "Readings".
+ */
+#ifndef VPIC_H
+#define VPIC_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  VPIC_OK = 0,
+  VPIC_ERR_INVALID = -1,     /* bad argument (null, misaligned, out of range) */
+  VPIC_ERR_CAPACITY = -2,    /* a caller buffer is too small (movers, np, ws) */
+  VPIC_ERR_CUDA = -3,        /* a CUDA runtime call failed */
+  VPIC_ERR_NCCL = -4,        /* an NCCL call failed */
+  VPIC_ERR_UNSUPPORTED = -5  /* wrong device (not sm_100) or feature absent */
+} vpic_status;
+
+/* Particle boundary condition per face (faces ordered -x,-y,-z,+x,+y,+z).
+ * PERIODIC: the particle passes into the block owned by nbr_rank[face]
+ * (a local wrap when nbr_rank[face] == the caller's rank).  REFLECT: the
+ * momentum and remaining displacement along the face normal are negated.
+ * ABSORB: the particle is removed after depositing up to the face. */
+enum { VPIC_BC_PERIODIC = 0, VPIC_BC_REFLECT = 1, VPIC_BC_ABSORB = 2 };
+
+/* Sort orders: standard classification by voxel, strided (Alg. 1,
+ * P:117-139), tiled strided (Alg. 2), none (input order kept;
+ * the paper's "random" order when the input is shuffled, Fig. 7). */
+enum { VPIC_SORT_STANDARD = 0, VPIC_SORT_STRIDED = 1, VPIC_SORT_TILED_STRIDED = 2,
+       VPIC_SORT_NONE = 3 };
+
+/* Context options (vpic_ctx_set_option). */
+enum {
+  /* advance_p arithmetic: 0 = FAST (FMA, fast rsqrt/div; within the oracle
+   * tolerances), 1 = IEEE (no FMA contraction, correctly rounded div/sqrt:
+   * bit-identical to the serial oracle). Default 0. */
+  VPIC_OPT_MATH = 0,
+  /* current scatter strategy: 0 = AUTO, 1 = LANE (3 x red.global.add.v4.f32 per
+   * streak), 2 = WARP (same-voxel contributions reduced across the warp with
+   * shuffles before red.global; falls back to LANE for scattered warps).
+   * Default AUTO (= WARP). */
+  VPIC_OPT_DEPOSIT = 1,
+  /* default TileSz for VPIC_SORT_TILED_STRIDED when tile_sz == 0.  Default
+   * 3 x (#SMs) x 128 ("three times the number of GPU cores"). */
+  VPIC_OPT_TILE_SZ = 2,
+  /* advance_p kernel variant: 0 = AUTO, 1 = direct global loads,
+   * 2 = TMA bulk-copy pipeline (particles staged through shared memory). */
+  VPIC_OPT_ADVANCE_KERNEL = 3
+};
+
+typedef struct {
+  int32_t nx, ny, nz;          /* local interior cells (>= 1 each) */
+  float dx, dy, dz, dt, cvac;  /* cell size, time step, speed of light */
+  int32_t pbc[6];              /* VPIC_BC_* per face */
+  int32_t nbr_rank[6];         /* rank owning the adjacent block (PERIODIC faces) */
+  int32_t gx0, gy0, gz0;       /* global offset of this block (cells; informational) */
+} vpic_grid_t;
+
+typedef struct { float dx, dy, dz; int32_t i; float ux, uy, uz, w; } vpic_particle_t; /* 32 B */
+typedef struct { float dispx, dispy, dispz; int32_t idx; } vpic_mover_t;              /* 16 B */
+typedef struct vpic_ctx vpic_ctx;
+
+/* ------------------------------------------------------------- context -- */
+
+/* NCCL unique id for a multi-GPU context (host call, rank 0 only; the caller
+ * broadcasts the 128 bytes, e.g. with torch.distributed). */
+int vpic_get_unique_id(uint8_t uid[128]);
+
+/* Create a context for one rank on CUDA device `device` (the caller has made
+ * it current or it is made current here).  nranks == 1: uid may be NULL, every
+ * PERIODIC face must have nbr_rank == rank.  nranks > 1: uid from
+ * vpic_get_unique_id; the call is collective over the nranks processes.
+ * Fails with VPIC_ERR_UNSUPPORTED on a device that is not compute capability
+ * 10.0 (the library holds sm_100a code only). */
+int vpic_ctx_create(vpic_ctx **ctx, const vpic_grid_t *g, int rank, int nranks,
+                    const uint8_t *uid, int device);
+int vpic_ctx_destroy(vpic_ctx *ctx);
+int vpic_ctx_set_option(vpic_ctx *ctx, int option, int64_t value);
+/* info[0]=#SMs, [1]=default tile size, [2]=nv, [3]=rank, [4]=nranks,
+ * [5]=L2 bytes, [6]=math mode, [7]=deposit mode. */
+int vpic_ctx_info(const vpic_ctx *ctx, int64_t info[8]);
+const char *vpic_status_string(int status);
+/* Number of CUDA kernels this process has launched through the library
+ * (all contexts; memsets and copies excluded).  Host call, never fails. */
+int64_t vpic_kernel_launches(void);
+
+/* ------------------------------------------------------ (a1-a4) sort -- */
+
+/* Bytes of device workspace vpic_sort_particles needs for np particles. */
+size_t vpic_sort_workspace_bytes(const vpic_ctx *ctx, int64_t np, int order);
+
+/* Sort particles by voxel key ("VPIC sorts particles according to the cell
+ * index") into `order`, out of place: p_out[j] = p_in[perm[j]].
+ * STANDARD = stable by voxel (reading R8).  STRIDED = Alg. 1: new key
+ * (k - min_k) + r (max_k + 1).  TILED_STRIDED = Alg. 2: new key
+ * floor(k/T) T max_r + r T + (k - min_k), T = tile_sz (0: context default).
+ * The rank r of a particle among equal keys is the number of EARLIER input
+ * particles with the same key (reading R1: deterministic, stable), so keys,
+ * counts and permutation are bit-reproducible.
+ *   p_in, p_out     [np] particles (must not overlap);
+ *   ws, ws_bytes    device workspace, >= vpic_sort_workspace_bytes();
+ *   voxel_counts    [nv] int32 out, nullable: particles per voxel;
+ *   new_keys        [np] int64 out, nullable: adjusted key of INPUT particle i
+ *                   (the raw key for STANDARD / NONE);
+ *   perm            [np] int64 out, nullable.
+ * np == 0 is valid (nothing enqueued except zeroing voxel_counts).  Keys
+ * outside [0, nv) are undefined behaviour (not checked on device). */
+int vpic_sort_particles(vpic_ctx *ctx, const vpic_particle_t *p_in, vpic_particle_t *p_out,
+                        int64_t np, int order, int64_t tile_sz, void *ws, size_t ws_bytes,
+                        int32_t *voxel_counts, int64_t *new_keys, int64_t *perm,
+                        void *stream);
+
+/* ---------------------------------------------------- (a5) interpolator -- */
+
+/* Fill the +x/+y/+z ghost planes of fields (locally periodic faces: copy of
+ * plane 1; remote faces: received from the neighbour over NCCL) in
+ * place, then write interp[v] for every interior voxel v (ghost voxels of
+ * interp are left untouched).  Ghost planes of REFLECT/ABSORB faces are the
+ * caller's. */
+int vpic_load_interpolator(vpic_ctx *ctx, float *fields, float *interp, void *stream);
+
+/* ------------------------------------------------ (a6) clear accumulator -- */
+int vpic_clear_accumulator(vpic_ctx *ctx, float *acc, void *stream);
+
+/* ----------------------------------------------- (a7-a11) particle push -- */
+
+/* One time step of np particles of one species (charge q, mass m): gather E
+ * and cB from interp at each particle, relativistic Boris push, move with cell
+ * crossing, charge-conserving current scatter into acc ("gather phase, atomic
+ * scatter phase, and additional physics computations").  acc is
+ * ACCUMULATED into (clear it once per step, before the first species).
+ * Particles are updated in place.  A particle that reaches a REMOTE or ABSORB
+ * face stops there (offset exactly +-1 on the face, p.i = 8*voxel + face) and
+ * appends a mover {remaining displacement, index} at movers[atomic n_movers++];
+ * the append order is unspecified.
+ *   n_movers   device int64, in/out (not reset by this call);
+ *   flags      device int32, nullable: bit 0 set if a mover was dropped
+ *              because *n_movers reached max_movers. */
+int vpic_advance_p(vpic_ctx *ctx, float q, float m, vpic_particle_t *p, int64_t np,
+                   const float *interp, float *acc, vpic_mover_t *movers, int64_t max_movers,
+                   int64_t *n_movers, int32_t *flags, void *stream);
+
+/* ------------------------------------------------------ (a12) unload -- */
+
+/* jf on every edge of voxels 1..n+1 from the 4 accumulators sharing it,
+ * times c_axis = 1/(4 dA dt); shared boundary planes summed (locally periodic
+ * axes: folded; remote faces: summed with the neighbour over NCCL) and the
+ * n+1 ghost copies made equal to plane 1.  jf is overwritten. */
+int vpic_unload_accumulator(vpic_ctx *ctx, const float *acc, float *jf, void *stream);
+
+/* ---------------------------------------------------- (a13) exchange -- */
+
+/* Finish the movers produced by vpic_advance_p for one species: particles on
+ * REMOTE faces are sent to the neighbour rank (NCCL send/recv, up to three
+ * rounds for corner crossings, "non-blocking point-to-point with up to six
+ * neighbors" P:55), received particles continue their move (depositing into
+ * acc) and are appended; absorbed and departed particles are removed by
+ * back-filling from the end.  *np (HOST) is updated.  SYNCHRONISES `stream`
+ * (it reads mover counts).  Fails with VPIC_ERR_CAPACITY if the arrivals would
+ * exceed max_np. */
+int vpic_migrate_particles(vpic_ctx *ctx, float q, float m, vpic_particle_t *p, int64_t *np,
+                           int64_t max_np, vpic_mover_t *movers, const int64_t *n_movers,
+                           float *acc, void *stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* VPIC_H */

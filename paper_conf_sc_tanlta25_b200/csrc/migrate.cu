@@ -1,0 +1,388 @@
+// Particle boundary handling and the multi-GPU exchange (row a13 of SURVEY.md
+// §8(a)): particle migration across rank faces ("Most MPI communication in
+// VPIC is non-blocking point-to-point with up to six neighbors", PAPER.md:55;
+// "exchanging particles"), the E/cB ghost-plane halo and the jf
+// shared-plane reduction.  Transport: NCCL send/recv (NVLink / NVSwitch) in
+// grouped calls; one process per GPU.
+#include <nccl.h>
+
+#include <algorithm>
+#include <vector>
+
+#include "vpic_internal.cuh"
+
+namespace vpic {
+
+struct Exchange {
+  ncclComm_t comm = nullptr;
+  // migration buffers (48-B records: particle + remaining displacement)
+  float4 *send = nullptr;   // [6][send_cap][3]
+  float4 *recv = nullptr;   // [recv_cap][3]
+  int64_t send_cap = 0, recv_cap = 0;
+  int64_t *d_cnt = nullptr; // [0..5] send counts, [6..11] recv counts
+  vpic_mover_t *mv_arr = nullptr, *mv_next = nullptr;  // arrivals' movers, next round's
+  int64_t mv_arr_cap = 0, mv_next_cap = 0;
+  // plane buffers for halo / jf reduction
+  float *plane_send = nullptr, *plane_recv = nullptr;
+  size_t plane_bytes = 0;
+};
+
+namespace {
+
+constexpr int OPP[6] = {3, 4, 5, 0, 1, 2};
+
+#define CKC(x) do { cudaError_t e_ = (x); if (e_ != cudaSuccess) return VPIC_ERR_CUDA; } while (0)
+#define CKN(x) do { ncclResult_t r_ = (x); if (r_ != ncclSuccess) return VPIC_ERR_NCCL; } while (0)
+
+struct Ptrs6 { float4 *p[6]; };
+
+// Classify the movers of this round: every mover's particle leaves this rank
+// (remote face: packed for the neighbour with its entry voxel and flipped
+// offset; absorb face: dropped).  Its slot becomes a hole.
+__global__ void k_pack_movers(const GridK g, const vpic_particle_t *__restrict__ p,
+                              const vpic_mover_t *__restrict__ mv, int64_t M, float4 *__restrict__ send,
+                              int64_t send_cap, int64_t *__restrict__ send_cnt,
+                              uint32_t *__restrict__ holes, int32_t *__restrict__ flags) {
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < M;
+       k += (int64_t)gridDim.x * blockDim.x) {
+    const vpic_mover_t m = mv[k];
+    holes[k] = (uint32_t)m.idx;
+    vpic_particle_t q = p[m.idx];
+    const int face = q.i & 7;
+    const int32_t v = q.i >> 3;
+    if (g.face_kind[face] != FACE_REMOTE) continue;  // absorbed
+    int x = v % g.sx, y = (v / g.sx) % g.sy, z = v / g.sxy;
+    const int axis = face % 3;
+    const bool plus = face >= 3;
+    if (axis == 0) { x = plus ? 1 : g.nx; q.dx = -q.dx; }
+    else if (axis == 1) { y = plus ? 1 : g.ny; q.dy = -q.dy; }
+    else { z = plus ? 1 : g.nz; q.dz = -q.dz; }
+    q.i = x + g.sx * (y + g.sy * z);
+    const unsigned long long slot = atomicAdd(reinterpret_cast<unsigned long long *>(send_cnt + face), 1ull);
+    if ((int64_t)slot >= send_cap) { atomicOr(flags, 2); continue; }
+    float4 *r = send + 3 * ((int64_t)face * send_cap + (int64_t)slot);
+    r[0] = make_float4(q.dx, q.dy, q.dz, __int_as_float(q.i));
+    r[1] = make_float4(q.ux, q.uy, q.uz, q.w);
+    r[2] = make_float4(m.dispx, m.dispy, m.dispz, 0.0f);
+  }
+}
+
+// Back-fill the H holes (distinct indices < np) with the surviving particles
+// of the tail [np-H, np).  scratch: 3*H + 2 ints.
+__global__ void k_mark_tail(const uint32_t *__restrict__ holes, int64_t H, int64_t np_new,
+                            uint32_t *__restrict__ tail_dead, uint32_t *__restrict__ low,
+                            unsigned long long *__restrict__ nlow) {
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < H;
+       k += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t h = holes[k];
+    if (h >= np_new) tail_dead[h - np_new] = 1;
+    else low[atomicAdd(nlow, 1ull)] = (uint32_t)h;
+  }
+}
+__global__ void k_tail_survivors(const uint32_t *__restrict__ tail_dead, int64_t H, int64_t np_new,
+                                 uint32_t *__restrict__ surv, unsigned long long *__restrict__ nsurv) {
+  for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < H;
+       j += (int64_t)gridDim.x * blockDim.x)
+    if (!tail_dead[j]) surv[atomicAdd(nsurv, 1ull)] = (uint32_t)(np_new + j);
+}
+__global__ void k_backfill(vpic_particle_t *__restrict__ p, const uint32_t *__restrict__ low,
+                           const uint32_t *__restrict__ surv, int64_t n) {
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n;
+       k += (int64_t)gridDim.x * blockDim.x)
+    p[low[k]] = p[surv[k]];
+}
+
+// Append arrivals and build their mover list (remaining displacement).
+__global__ void k_unpack(const float4 *__restrict__ recv, int64_t A, vpic_particle_t *__restrict__ p,
+                         int64_t np, vpic_mover_t *__restrict__ mv) {
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < A;
+       k += (int64_t)gridDim.x * blockDim.x) {
+    const float4 a = recv[3 * k], b = recv[3 * k + 1], d = recv[3 * k + 2];
+    float4 *dst = reinterpret_cast<float4 *>(p + np + k);
+    dst[0] = a;
+    dst[1] = b;
+    vpic_mover_t m;
+    m.dispx = d.x; m.dispy = d.y; m.dispz = d.z; m.idx = (int32_t)(np + k);
+    mv[k] = m;
+  }
+}
+
+// ---- planes: (axis, index) plane of an array of nv records of `w` floats,
+// over the full extent of the other two axes (ghosts included).
+__global__ void k_plane_copy(const GridK g, int axis, int idx, float *__restrict__ a, int w,
+                             float *__restrict__ buf, int mode /*0 pack, 1 unpack, 2 add*/) {
+  const int sz = g.nv / ((int64_t)g.sx * g.sy);
+  const int e0 = axis == 0 ? g.sy : g.sx;
+  const int e1 = axis == 2 ? g.sy : sz;
+  const int64_t n = (int64_t)e0 * e1 * w;
+  for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < n;
+       t += (int64_t)gridDim.x * blockDim.x) {
+    const int c = (int)(t % w);
+    const int64_t r = t / w;
+    const int u = (int)(r % e0), vv = (int)(r / e0);
+    int x, y, z;
+    if (axis == 0) { x = idx; y = u; z = vv; }
+    else if (axis == 1) { x = u; y = idx; z = vv; }
+    else { x = u; y = vv; z = idx; }
+    float *e = a + (int64_t)w * (x + (int64_t)g.sx * (y + (int64_t)g.sy * z)) + c;
+    if (mode == 0) buf[t] = *e;
+    else if (mode == 1) *e = buf[t];
+    else *e += buf[t];
+  }
+}
+
+unsigned blocks_for(int64_t n) {
+  int64_t b = (n + 255) / 256;
+  return (unsigned)std::max<int64_t>(1, std::min<int64_t>(b, 148 * 16));
+}
+
+int ensure(void **ptr, int64_t *cap, int64_t need, size_t rec_bytes) {
+  if (need <= *cap) return VPIC_OK;
+  if (*ptr) cudaFree(*ptr);
+  int64_t nc = std::max<int64_t>(need, *cap * 2);
+  nc = std::max<int64_t>(nc, 4096);
+  if (cudaMalloc(ptr, (size_t)nc * rec_bytes) != cudaSuccess) { *ptr = nullptr; *cap = 0; return VPIC_ERR_CUDA; }
+  *cap = nc;
+  return VPIC_OK;
+}
+
+int ensure_plane(Exchange *ex, size_t bytes) {
+  if (bytes <= ex->plane_bytes) return VPIC_OK;
+  if (ex->plane_send) cudaFree(ex->plane_send);
+  if (ex->plane_recv) cudaFree(ex->plane_recv);
+  if (cudaMalloc(&ex->plane_send, bytes) != cudaSuccess) return VPIC_ERR_CUDA;
+  if (cudaMalloc(&ex->plane_recv, bytes) != cudaSuccess) return VPIC_ERR_CUDA;
+  ex->plane_bytes = bytes;
+  return VPIC_OK;
+}
+
+// Scratch of the context used for hole filling (grown on demand).
+int ctx_scratch(vpic_ctx *c, size_t bytes) {
+  if (bytes <= c->scratch_bytes) return VPIC_OK;
+  if (c->scratch) cudaFree(c->scratch);
+  c->scratch = nullptr;
+  c->scratch_bytes = 0;
+  if (cudaMalloc(&c->scratch, bytes) != cudaSuccess) return VPIC_ERR_CUDA;
+  c->scratch_bytes = bytes;
+  return VPIC_OK;
+}
+
+int remove_holes(vpic_ctx *c, vpic_particle_t *p, int64_t np, const uint32_t *holes, int64_t H,
+                 cudaStream_t s) {
+  if (H == 0) return VPIC_OK;
+  const int64_t np_new = np - H;
+  uint32_t *sc = static_cast<uint32_t *>(c->scratch) + H;  // after the hole list
+  uint32_t *tail_dead = sc, *low = sc + H, *surv = sc + 2 * H;
+  unsigned long long *cnt = reinterpret_cast<unsigned long long *>(c->d_count + 2);
+  CKC(cudaMemsetAsync(tail_dead, 0, 4 * (size_t)H, s));
+  CKC(cudaMemsetAsync(cnt, 0, 16, s));
+  k_mark_tail<<<blocks_for(H), 256, 0, s>>>(holes, H, np_new, tail_dead, low, cnt); note_launch();
+  k_tail_survivors<<<blocks_for(H), 256, 0, s>>>(tail_dead, H, np_new, surv, cnt + 1); note_launch();
+  int64_t h_low = 0;
+  CKC(cudaMemcpyAsync(&h_low, cnt, 8, cudaMemcpyDeviceToHost, s));
+  CKC(cudaStreamSynchronize(s));
+  if (h_low) { k_backfill<<<blocks_for(h_low), 256, 0, s>>>(p, low, surv, h_low); note_launch(); }
+  return cudaGetLastError() == cudaSuccess ? VPIC_OK : VPIC_ERR_CUDA;
+}
+
+}  // namespace
+
+int exchange_create(vpic_ctx *c, const uint8_t *uid) {
+  Exchange *ex = new Exchange();
+  ncclUniqueId id;
+  static_assert(sizeof(id.internal) == 128, "nccl unique id size");
+  std::copy(uid, uid + 128, id.internal);
+  if (ncclCommInitRank(&ex->comm, c->nranks, id, c->rank) != ncclSuccess) {
+    delete ex;
+    return VPIC_ERR_NCCL;
+  }
+  if (cudaMalloc(&ex->d_cnt, 16 * sizeof(int64_t)) != cudaSuccess) {
+    ncclCommDestroy(ex->comm);
+    delete ex;
+    return VPIC_ERR_CUDA;
+  }
+  c->ex = ex;
+  return VPIC_OK;
+}
+
+void exchange_destroy(vpic_ctx *c) {
+  Exchange *ex = c->ex;
+  if (!ex) return;
+  if (ex->comm) ncclCommDestroy(ex->comm);
+  cudaFree(ex->send);
+  cudaFree(ex->recv);
+  cudaFree(ex->d_cnt);
+  cudaFree(ex->plane_send);
+  cudaFree(ex->plane_recv);
+  cudaFree(ex->mv_arr);
+  cudaFree(ex->mv_next);
+  delete ex;
+  c->ex = nullptr;
+}
+
+// Up to 3 rounds: pack movers per face, exchange counts, exchange records,
+// remove departed / absorbed particles, append arrivals, continue their move.
+int migrate(vpic_ctx *c, float qsp, float msp, vpic_particle_t *p, int64_t *np_io, int64_t max_np,
+            vpic_mover_t *movers, const int64_t *n_movers, float *acc, cudaStream_t s) {
+  (void)msp;
+  int64_t M = 0;
+  CKC(cudaMemcpyAsync(&M, n_movers, 8, cudaMemcpyDeviceToHost, s));
+  CKC(cudaStreamSynchronize(s));
+  int64_t np = *np_io;
+  if (M > np) return VPIC_ERR_INVALID;
+  int32_t *d_flags = reinterpret_cast<int32_t *>(c->d_count + 1);
+  CKC(cudaMemsetAsync(d_flags, 0, 4, s));
+  Exchange *ex = c->ex;
+  const vpic_mover_t *cur = movers;
+  const int rounds = ex ? 3 : 1;
+  for (int round = 0; round <= rounds; ++round) {
+    const bool exchange = ex && round < rounds;
+    if (!exchange && M == 0) break;
+    const int64_t Mpad = std::max<int64_t>(M, 1);
+    if (int rc = ctx_scratch(c, 16 * (size_t)Mpad + 64)) return rc;
+    uint32_t *holes = static_cast<uint32_t *>(c->scratch);
+    int64_t *cnt = ex ? ex->d_cnt : c->d_count + 3;
+    if (exchange) {
+      int64_t tot = ex->send_cap * 6;
+      if (int rc = ensure(reinterpret_cast<void **>(&ex->send), &tot, 6 * Mpad, 48)) return rc;
+      ex->send_cap = tot / 6;
+    }
+    CKC(cudaMemsetAsync(cnt, 0, (ex ? 12 : 1) * sizeof(int64_t), s));
+    if (M > 0) {
+      k_pack_movers<<<blocks_for(M), 256, 0, s>>>(c->gk, p, cur, M, exchange ? ex->send : nullptr,
+                                                   exchange ? ex->send_cap : 0, cnt, holes, d_flags); note_launch();
+      CKC(cudaGetLastError());
+    }
+    int64_t sent[6] = {0, 0, 0, 0, 0, 0}, rcvd[6] = {0, 0, 0, 0, 0, 0}, A = 0;
+    if (exchange) {
+      // counts: one int64 per face to nbr_rank[f]; the neighbour's count for
+      // its face f arrives on my face OPP[f] (posting order matches per pair)
+      CKN(ncclGroupStart());
+      for (int f = 0; f < 6; ++f)
+        if (c->gk.face_kind[f] == FACE_REMOTE)
+          CKN(ncclSend(cnt + f, 1, ncclInt64, c->g.nbr_rank[f], ex->comm, s));
+      for (int f = 0; f < 6; ++f) {
+        const int o = OPP[f];
+        if (c->gk.face_kind[o] == FACE_REMOTE)
+          CKN(ncclRecv(cnt + 6 + o, 1, ncclInt64, c->g.nbr_rank[o], ex->comm, s));
+      }
+      CKN(ncclGroupEnd());
+      int64_t h[12];
+      CKC(cudaMemcpyAsync(h, cnt, sizeof(h), cudaMemcpyDeviceToHost, s));
+      CKC(cudaStreamSynchronize(s));
+      for (int f = 0; f < 6; ++f) {
+        sent[f] = h[f];
+        rcvd[f] = h[6 + f];
+        A += rcvd[f];
+        if (sent[f] > ex->send_cap) return VPIC_ERR_CAPACITY;
+      }
+      if (int rc = ensure(reinterpret_cast<void **>(&ex->recv), &ex->recv_cap, std::max<int64_t>(A, 1), 48))
+        return rc;
+      float4 *rptr[6];
+      int64_t roff = 0;
+      for (int f = 0; f < 6; ++f) { rptr[f] = ex->recv + 3 * roff; roff += rcvd[f]; }
+      CKN(ncclGroupStart());
+      for (int f = 0; f < 6; ++f)
+        if (c->gk.face_kind[f] == FACE_REMOTE)
+          CKN(ncclSend(ex->send + 3 * (int64_t)f * ex->send_cap, (size_t)sent[f] * 12, ncclFloat32,
+                       c->g.nbr_rank[f], ex->comm, s));
+      for (int f = 0; f < 6; ++f) {
+        const int o = OPP[f];
+        if (c->gk.face_kind[o] == FACE_REMOTE)
+          CKN(ncclRecv(rptr[o], (size_t)rcvd[o] * 12, ncclFloat32, c->g.nbr_rank[o], ex->comm, s));
+      }
+      CKN(ncclGroupEnd());
+    }
+    // every mover's particle has left this rank (sent or absorbed)
+    if (int rc = remove_holes(c, p, np, holes, M, s)) return rc;
+    np -= M;
+    M = 0;
+    if (!exchange) break;
+    if (np + A > max_np) return VPIC_ERR_CAPACITY;
+    if (A > 0) {
+      if (int rc = ensure(reinterpret_cast<void **>(&ex->mv_arr), &ex->mv_arr_cap, A, 16)) return rc;
+      if (int rc = ensure(reinterpret_cast<void **>(&ex->mv_next), &ex->mv_next_cap, A, 16)) return rc;
+      k_unpack<<<blocks_for(A), 256, 0, s>>>(ex->recv, A, p, np, ex->mv_arr); note_launch();
+      CKC(cudaGetLastError());
+      int64_t *d_next = c->d_count + 3;
+      CKC(cudaMemsetAsync(d_next, 0, 8, s));
+      cudaError_t e = (c->math == MATH_IEEE)
+                          ? launch_move_movers_ieee(c, qsp, p, ex->mv_arr, A, acc, ex->mv_next, A, d_next, d_flags, s)
+                          : launch_move_movers_fast(c, qsp, p, ex->mv_arr, A, acc, ex->mv_next, A, d_next, d_flags, s);
+      CKC(e);
+      CKC(cudaMemcpyAsync(&M, d_next, 8, cudaMemcpyDeviceToHost, s));
+      CKC(cudaStreamSynchronize(s));
+      np += A;
+      cur = ex->mv_next;
+    }
+  }
+  int32_t hflag = 0;
+  CKC(cudaMemcpyAsync(&hflag, d_flags, 4, cudaMemcpyDeviceToHost, s));
+  CKC(cudaStreamSynchronize(s));
+  *np_io = np;
+  if (hflag) return VPIC_ERR_CAPACITY;
+  return VPIC_OK;
+}
+
+// E/cB ghost planes from the neighbours: axis by axis, my plane 1 goes to the
+// -face neighbour, whose plane n+1 it fills (edges/corners propagate).
+int halo_fields(vpic_ctx *c, float *fields, cudaStream_t s) {
+  Exchange *ex = c->ex;
+  const GridK &g = c->gk;
+  const int sz = g.nz + 2;
+  const size_t maxplane = (size_t)std::max({(int64_t)g.sy * sz, (int64_t)g.sx * sz, (int64_t)g.sx * g.sy}) * 8 * 4;
+  if (int rc = ensure_plane(ex, maxplane)) return rc;
+  for (int axis = 0; axis < 3; ++axis) {
+    if (c->periodic_local[axis]) continue;
+    const int fm = axis, fp = axis + 3;
+    const bool send_m = g.face_kind[fm] == FACE_REMOTE, recv_p = g.face_kind[fp] == FACE_REMOTE;
+    if (!send_m && !recv_p) continue;
+    const int n = axis == 0 ? g.nx : (axis == 1 ? g.ny : g.nz);
+    const int64_t cnt = (axis == 0 ? (int64_t)g.sy * sz : axis == 1 ? (int64_t)g.sx * sz : (int64_t)g.sx * g.sy) * 8;
+    if (send_m) { k_plane_copy<<<blocks_for(cnt), 256, 0, s>>>(g, axis, 1, fields, 8, ex->plane_send, 0); note_launch(); }
+    CKN(ncclGroupStart());
+    if (send_m) CKN(ncclSend(ex->plane_send, cnt, ncclFloat32, c->g.nbr_rank[fm], ex->comm, s));
+    if (recv_p) CKN(ncclRecv(ex->plane_recv, cnt, ncclFloat32, c->g.nbr_rank[fp], ex->comm, s));
+    CKN(ncclGroupEnd());
+    if (recv_p) { k_plane_copy<<<blocks_for(cnt), 256, 0, s>>>(g, axis, n + 1, fields, 8, ex->plane_recv, 1); note_launch(); }
+    CKC(cudaGetLastError());
+  }
+  return VPIC_OK;
+}
+
+// jf shared planes: my plane n+1 partial sums belong to the +face neighbour's
+// plane 1 (added there); then the completed plane 1 is sent back to fill the
+// -face neighbour's plane n+1.  Axis by axis.
+int reduce_jf(vpic_ctx *c, float *jf, cudaStream_t s) {
+  Exchange *ex = c->ex;
+  const GridK &g = c->gk;
+  const int sz = g.nz + 2;
+  const size_t maxplane = (size_t)std::max({(int64_t)g.sy * sz, (int64_t)g.sx * sz, (int64_t)g.sx * g.sy}) * 4 * 4;
+  if (int rc = ensure_plane(ex, maxplane)) return rc;
+  for (int axis = 0; axis < 3; ++axis) {
+    if (c->periodic_local[axis]) continue;
+    const int fm = axis, fp = axis + 3;
+    const bool rm = g.face_kind[fm] == FACE_REMOTE, rp = g.face_kind[fp] == FACE_REMOTE;
+    if (!rm && !rp) continue;
+    const int n = axis == 0 ? g.nx : (axis == 1 ? g.ny : g.nz);
+    const int64_t cnt = (axis == 0 ? (int64_t)g.sy * sz : axis == 1 ? (int64_t)g.sx * sz : (int64_t)g.sx * g.sy) * 4;
+    // phase 1: plane n+1 -> +neighbour, add into plane 1
+    if (rp) { k_plane_copy<<<blocks_for(cnt), 256, 0, s>>>(g, axis, n + 1, jf, 4, ex->plane_send, 0); note_launch(); }
+    CKN(ncclGroupStart());
+    if (rp) CKN(ncclSend(ex->plane_send, cnt, ncclFloat32, c->g.nbr_rank[fp], ex->comm, s));
+    if (rm) CKN(ncclRecv(ex->plane_recv, cnt, ncclFloat32, c->g.nbr_rank[fm], ex->comm, s));
+    CKN(ncclGroupEnd());
+    if (rm) { k_plane_copy<<<blocks_for(cnt), 256, 0, s>>>(g, axis, 1, jf, 4, ex->plane_recv, 2); note_launch(); }
+    // phase 2: plane 1 -> -neighbour's plane n+1
+    if (rm) { k_plane_copy<<<blocks_for(cnt), 256, 0, s>>>(g, axis, 1, jf, 4, ex->plane_send, 0); note_launch(); }
+    CKN(ncclGroupStart());
+    if (rm) CKN(ncclSend(ex->plane_send, cnt, ncclFloat32, c->g.nbr_rank[fm], ex->comm, s));
+    if (rp) CKN(ncclRecv(ex->plane_recv, cnt, ncclFloat32, c->g.nbr_rank[fp], ex->comm, s));
+    CKN(ncclGroupEnd());
+    if (rp) { k_plane_copy<<<blocks_for(cnt), 256, 0, s>>>(g, axis, n + 1, jf, 4, ex->plane_recv, 1); note_launch(); }
+    CKC(cudaGetLastError());
+  }
+  return VPIC_OK;
+}
+
+}  // namespace vpic

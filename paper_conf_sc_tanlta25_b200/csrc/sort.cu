@@ -1,0 +1,552 @@
+// Hardware-targeted particle sort by voxel (rows a1-a4 of SURVEY.md §8(a)):
+// standard classification, strided (Alg. 1) and
+// tiled strided (Alg. 2).
+//
+// B200 design: the paper adjusts keys in O(N) and then calls
+// a generic sort_by_key.  Here every order is produced by stable LSD
+// counting passes with no comparison sort and no nondeterministic atomics:
+//   standard      = stable radix sort of (voxel, index) pairs, 2 passes of
+//                   <= 13-bit digits (chained-scan / decoupled look-back);
+//   strided       = standard, then one stable counting pass by the rank
+//                   r = pos - offset[voxel]        (lexicographic (r, k));
+//   tiled strided = standard, then one stable counting pass by
+//                   (floor(k/T) - floor(min_k/T)) * max_r + r   (lexicographic
+//                   (floor(k/T), r, k)).
+// The rank of a particle among equal keys is its stable rank (reading R1), so
+// the result equals Alg. 1/2 with the atomic_fetch_add loop run in input
+// order: keys, counts and permutation are bit-exact against the oracle.
+#include <algorithm>
+
+#include "vpic_internal.cuh"
+
+namespace vpic {
+namespace {
+
+constexpr int NT = 256;             // threads per radix CTA
+constexpr int NW = NT / 32;         // warps
+constexpr int IPT = 32;             // items per thread
+constexpr int TILE = NT * IPT;      // 8192 elements per tile
+constexpr int MAX_BITS = 13;        // digit width limit (smem: NW * 2^13 * 2 B = 128 KB)
+constexpr int MAX_PASSES = 3;
+constexpr unsigned FULL = 0xffffffffu;
+
+constexpr unsigned long long FLAG_AGG = 1ull << 62;
+constexpr unsigned long long FLAG_INC = 2ull << 62;
+constexpr unsigned long long VAL_MASK = (1ull << 40) - 1;
+
+__device__ __forceinline__ void st_relaxed(unsigned long long *p, unsigned long long v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long ld_relaxed(const unsigned long long *p) {
+  unsigned long long v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ unsigned lanemask_lt() {
+  unsigned m;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+  return m;
+}
+
+struct PassDesc {
+  int shift[MAX_PASSES];
+  int bits[MAX_PASSES];
+  int npass;
+};
+
+// ---------------------------------------------------------------- a1 --
+// keys[i] = p_in[i].i ; digit histograms of every pass (warp-aggregated smem
+// counters, one global atomic per non-empty bin per CTA); optional raw
+// new_keys (STANDARD / NONE).
+__global__ void __launch_bounds__(256)
+k_keys_hist(const vpic_particle_t *__restrict__ p, int64_t n, uint32_t *__restrict__ keys,
+            PassDesc pd, uint32_t *__restrict__ ghist /*[MAX_PASSES][1<<MAX_BITS]*/,
+            int64_t *__restrict__ new_keys) {
+  extern __shared__ uint32_t sh[];  // [npass][1<<bits_q] (packed)
+  int off[MAX_PASSES];
+  int tot = 0;
+  for (int q = 0; q < pd.npass; ++q) { off[q] = tot; tot += 1 << pd.bits[q]; }
+  for (int i = threadIdx.x; i < tot; i += blockDim.x) sh[i] = 0;
+  __syncthreads();
+  const int lane = threadIdx.x & 31;
+  const int32_t *pi = reinterpret_cast<const int32_t *>(p) + 3;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t base = (int64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31); base < n;
+       base += stride) {
+    const int64_t i = base + lane;
+    const bool valid = i < n;
+    uint32_t k = 0;
+    if (valid) {
+      k = (uint32_t)__ldcs(pi + 8 * i);
+      keys[i] = k;
+      if (new_keys) new_keys[i] = (int64_t)k;
+    }
+    for (int q = 0; q < pd.npass; ++q) {
+      const uint32_t d = valid ? ((k >> pd.shift[q]) & ((1u << pd.bits[q]) - 1)) : 0xffffffffu;
+      const unsigned peers = __match_any_sync(FULL, d);
+      if (valid && (__ffs(peers) - 1) == lane) atomicAdd(&sh[off[q] + d], __popc(peers));
+    }
+  }
+  __syncthreads();
+  for (int q = 0; q < pd.npass; ++q)
+    for (int b = threadIdx.x; b < (1 << pd.bits[q]); b += blockDim.x) {
+      const uint32_t c = sh[off[q] + b];
+      if (c) atomicAdd(&ghist[q * (1 << MAX_BITS) + b], c);
+    }
+}
+
+// Exclusive scan of each pass's digit histogram (one CTA per pass).
+__global__ void k_scan_hist(const uint32_t *__restrict__ ghist, uint32_t *__restrict__ goff,
+                            PassDesc pd) {
+  const int q = blockIdx.x;
+  if (q >= pd.npass) return;
+  const int nb = 1 << pd.bits[q];
+  __shared__ uint32_t part[1024];
+  const uint32_t *h = ghist + q * (1 << MAX_BITS);
+  uint32_t *o = goff + q * (1 << MAX_BITS);
+  const int per = (nb + blockDim.x - 1) / blockDim.x;
+  const int b0 = threadIdx.x * per;
+  uint32_t s = 0;
+  for (int b = b0; b < min(nb, b0 + per); ++b) s += h[b];
+  part[threadIdx.x] = s;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t run = 0;
+    for (int t = 0; t < (int)blockDim.x; ++t) { const uint32_t x = part[t]; part[t] = run; run += x; }
+  }
+  __syncthreads();
+  uint32_t run = part[threadIdx.x];
+  for (int b = b0; b < min(nb, b0 + per); ++b) { o[b] = run; run += h[b]; }
+}
+
+// ---------------------------------------------------------------- a3/a4 --
+// One stable LSD counting pass over (key, val) with a 2^BITS-bucket digit.
+// Tiles are taken in order from an atomic ticket; each tile ranks its
+// elements stably (per-warp smem histograms, match_any within a warp),
+// publishes its per-digit count and resolves its global offset by decoupled
+// look-back over earlier tiles' status words (flag | count in one u64).
+template <int BITS>
+__global__ void __launch_bounds__(NT)
+k_radix_pass(const uint32_t *__restrict__ kin, const uint32_t *__restrict__ vin,
+             uint32_t *__restrict__ kout, uint32_t *__restrict__ vout, int64_t n, int shift,
+             const uint32_t *__restrict__ dig_off, unsigned long long *__restrict__ status,
+             unsigned int *__restrict__ tile_ctr) {
+  constexpr int NB = 1 << BITS;
+  extern __shared__ __align__(16) unsigned char smem[];
+  uint16_t *whist = reinterpret_cast<uint16_t *>(smem);                       // [NW][NB]
+  uint32_t *tpref = reinterpret_cast<uint32_t *>(smem + NW * NB * 2);          // [NB]
+  __shared__ unsigned int s_tile;
+  if (threadIdx.x == 0) s_tile = atomicAdd(tile_ctr, 1u);
+  for (int i = threadIdx.x; i < NW * NB / 2; i += NT) reinterpret_cast<uint32_t *>(whist)[i] = 0;
+  __syncthreads();
+  const int64_t tile = s_tile;
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t wbase = tile * TILE + (int64_t)w * 32 * IPT;
+
+  uint32_t key[IPT], val[IPT];
+  uint32_t rank[IPT / 2];  // two u16 ranks per register
+#pragma unroll
+  for (int j = 0; j < IPT; ++j) {
+    const int64_t i = wbase + j * 32 + lane;
+    const bool valid = i < n;
+    key[j] = valid ? __ldcs(kin + i) : 0u;
+    val[j] = valid ? (vin ? __ldcs(vin + i) : (uint32_t)i) : 0u;
+  }
+  const unsigned lt = lanemask_lt();
+  uint16_t *wh = whist + w * NB;
+#pragma unroll
+  for (int j = 0; j < IPT; ++j) {
+    const int64_t i = wbase + j * 32 + lane;
+    const bool valid = i < n;
+    const uint32_t d = valid ? ((key[j] >> shift) & (NB - 1)) : (uint32_t)NB;
+    const unsigned peers = __match_any_sync(FULL, d);
+    uint32_t cur = 0;
+    if (valid) cur = wh[d];
+    __syncwarp();
+    if (valid && (__ffs(peers) - 1) == lane) wh[d] = (uint16_t)(cur + __popc(peers));
+    __syncwarp();
+    const uint32_t r = cur + __popc(peers & lt);
+    if (j & 1) rank[j >> 1] |= r << 16; else rank[j >> 1] = r;
+  }
+  __syncthreads();
+  // per-digit: warp exclusive offsets, tile count, look-back
+  for (int b = threadIdx.x; b < NB; b += NT) {
+    uint32_t run = 0;
+#pragma unroll
+    for (int ww = 0; ww < NW; ++ww) {
+      const uint32_t c = whist[ww * NB + b];
+      whist[ww * NB + b] = (uint16_t)run;
+      run += c;
+    }
+    unsigned long long *st = status + tile * NB + b;
+    uint64_t excl = 0;
+    if (tile == 0) {
+      st_relaxed(st, FLAG_INC | run);
+    } else {
+      st_relaxed(st, FLAG_AGG | run);
+      int64_t t = tile - 1;
+      while (true) {
+        const unsigned long long s = ld_relaxed(status + t * NB + b);
+        const unsigned long long f = s & (3ull << 62);
+        if (f == 0) continue;
+        excl += s & VAL_MASK;
+        if (f == FLAG_INC) break;
+        --t;
+      }
+      st_relaxed(st, FLAG_INC | (excl + run));
+    }
+    tpref[b] = dig_off[b] + (uint32_t)excl;
+  }
+  __syncthreads();
+#pragma unroll
+  for (int j = 0; j < IPT; ++j) {
+    const int64_t i = wbase + j * 32 + lane;
+    if (i < n) {
+      const uint32_t d = (key[j] >> shift) & (NB - 1);
+      const uint32_t r = (j & 1) ? (rank[j >> 1] >> 16) : (rank[j >> 1] & 0xffffu);
+      const uint32_t pos = tpref[d] + whist[w * NB + d] + r;
+      if (kout) kout[pos] = key[j];
+      vout[pos] = val[j];
+    }
+  }
+}
+
+// ---------------------------------------------------------------- counts --
+// offs[k] = first standard-order position with key >= k, k in [0, nv]
+// (lower bound), from the sorted keys; every entry written exactly once.
+__global__ void k_offsets(const uint32_t *__restrict__ K, int64_t n, int64_t nv,
+                          uint32_t *__restrict__ offs) {
+  for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n;
+       j += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t prev = j == 0 ? -1 : (int64_t)K[j - 1];
+    const int64_t cur = K[j];
+    for (int64_t k = prev + 1; k <= cur; ++k) offs[k] = (uint32_t)j;
+    if (j == n - 1)
+      for (int64_t k = cur + 1; k <= nv; ++k) offs[k] = (uint32_t)n;
+  }
+}
+
+__global__ void k_counts(const uint32_t *__restrict__ offs, int64_t nv, int32_t *__restrict__ counts,
+                         unsigned int *__restrict__ max_r) {
+  unsigned int m = 0;
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < nv;
+       k += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t c = offs[k + 1] - offs[k];
+    if (counts) counts[k] = (int32_t)c;
+    m = max(m, c);
+  }
+  for (int o = 16; o; o >>= 1) m = max(m, __shfl_xor_sync(FULL, m, o));
+  if ((threadIdx.x & 31) == 0 && m) atomicMax(max_r, m);
+}
+
+// Rank-pass keys (strided: r; tiled: (chunk - chunk0) * max_r + r) with the
+// digit histograms of the following passes; optional Alg. 1/2 new keys
+// scattered to the INPUT index (perm_std[j]).
+__global__ void __launch_bounds__(256)
+k_rank_keys(const uint32_t *__restrict__ K, const uint32_t *__restrict__ perm_std,
+            const uint32_t *__restrict__ offs, int64_t n, int order, int64_t T, uint32_t max_r,
+            uint32_t *__restrict__ ckey, PassDesc pd, uint32_t *__restrict__ ghist,
+            int64_t *__restrict__ new_keys) {
+  extern __shared__ uint32_t sh[];
+  int off[MAX_PASSES];
+  int tot = 0;
+  for (int q = 0; q < pd.npass; ++q) { off[q] = tot; tot += 1 << pd.bits[q]; }
+  for (int i = threadIdx.x; i < tot; i += blockDim.x) sh[i] = 0;
+  __syncthreads();
+  const int lane = threadIdx.x & 31;
+  const int64_t min_k = K[0], max_k = K[n - 1];
+  const int64_t chunk0 = min_k / T;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t base = (int64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31); base < n;
+       base += stride) {
+    const int64_t j = base + lane;
+    const bool valid = j < n;
+    uint32_t ck = 0;
+    if (valid) {
+      const int64_t k = K[j];
+      const int64_t r = j - (int64_t)offs[k];
+      if (order == VPIC_SORT_STRIDED) {
+        ck = (uint32_t)r;
+        if (new_keys) new_keys[perm_std[j]] = (k - min_k) + r * (max_k + 1);
+      } else {
+        ck = (uint32_t)((k / T - chunk0) * (int64_t)max_r + r);
+        if (new_keys) new_keys[perm_std[j]] = (k / T) * (T * (int64_t)max_r) + r * T + (k - min_k);
+      }
+      ckey[j] = ck;
+    }
+    for (int q = 0; q < pd.npass; ++q) {
+      const uint32_t d = valid ? ((ck >> pd.shift[q]) & ((1u << pd.bits[q]) - 1)) : 0xffffffffu;
+      const unsigned peers = __match_any_sync(FULL, d);
+      if (valid && (__ffs(peers) - 1) == lane) atomicAdd(&sh[off[q] + d], __popc(peers));
+    }
+  }
+  __syncthreads();
+  for (int q = 0; q < pd.npass; ++q)
+    for (int b = threadIdx.x; b < (1 << pd.bits[q]); b += blockDim.x) {
+      const uint32_t c = sh[off[q] + b];
+      if (c) atomicAdd(&ghist[q * (1 << MAX_BITS) + b], c);
+    }
+}
+
+// ---------------------------------------------------------------- a4 --
+__global__ void __launch_bounds__(256)
+k_gather(const vpic_particle_t *__restrict__ pin, vpic_particle_t *__restrict__ pout,
+         const uint32_t *__restrict__ perm, int64_t n, int64_t *__restrict__ perm64) {
+  const float4 *src = reinterpret_cast<const float4 *>(pin);
+  float4 *dst = reinterpret_cast<float4 *>(pout);
+  for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < n;
+       t += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t s = perm[t];
+    const float4 a = __ldcs(src + 2 * (int64_t)s), b = __ldcs(src + 2 * (int64_t)s + 1);
+    __stcs(dst + 2 * t, a);
+    __stcs(dst + 2 * t + 1, b);
+    if (perm64) perm64[t] = s;
+  }
+}
+
+__global__ void k_iota64(int64_t *__restrict__ a, int64_t n) {
+  for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < n;
+       t += (int64_t)gridDim.x * blockDim.x)
+    a[t] = t;
+}
+
+__global__ void k_hist_voxels(const vpic_particle_t *__restrict__ p, int64_t n,
+                              int32_t *__restrict__ counts, int64_t *__restrict__ new_keys) {
+  const int32_t *pi = reinterpret_cast<const int32_t *>(p) + 3;
+  const int lane = threadIdx.x & 31;
+  for (int64_t base = (int64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31); base < n;
+       base += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t i = base + lane;
+    const bool valid = i < n;
+    const int32_t k = valid ? pi[8 * i] : -1;
+    if (valid && new_keys) new_keys[i] = k;
+    const unsigned peers = __match_any_sync(FULL, k);
+    if (valid && counts && (__ffs(peers) - 1) == lane) atomicAdd(&counts[k], __popc(peers));
+  }
+}
+
+// ------------------------------------------------------------ host side --
+struct WsLayout {
+  size_t keysA, keysB, valsA, valsB, offs, ghist, goff, status, ctr, misc, total;
+};
+
+inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+WsLayout layout(int64_t np, int64_t nv) {
+  WsLayout L{};
+  size_t o = 0;
+  auto take = [&](size_t bytes) { size_t r = o; o = align_up(o + bytes, 256); return r; };
+  const int64_t tiles = (np + TILE - 1) / TILE;
+  L.keysA = take(4 * (size_t)np);
+  L.keysB = take(4 * (size_t)np);
+  L.valsA = take(4 * (size_t)np);
+  L.valsB = take(4 * (size_t)np);
+  L.offs = take(4 * (size_t)(nv + 1));
+  L.ghist = take(4 * (size_t)MAX_PASSES * (1 << MAX_BITS));
+  L.goff = take(4 * (size_t)MAX_PASSES * (1 << MAX_BITS));
+  L.status = take(8 * (size_t)std::max<int64_t>(tiles, 1) * (1 << MAX_BITS));
+  L.ctr = take(4 * MAX_PASSES);
+  L.misc = take(64);
+  L.total = o;
+  return L;
+}
+
+int bits_for(uint64_t max_value) {  // bits needed to hold values 0..max_value
+  int b = 0;
+  while (b < 40 && (max_value >> b)) ++b;
+  return std::max(b, 1);
+}
+
+PassDesc make_passes(int nbits) {
+  PassDesc pd{};
+  pd.npass = (nbits + MAX_BITS - 1) / MAX_BITS;
+  if (pd.npass < 1) pd.npass = 1;
+  int rem = nbits, sh = 0;
+  for (int q = 0; q < pd.npass; ++q) {
+    const int b = (rem + (pd.npass - q) - 1) / (pd.npass - q);
+    pd.bits[q] = std::max(b, 1);
+    pd.shift[q] = sh;
+    sh += b;
+    rem -= b;
+  }
+  return pd;
+}
+
+template <int BITS>
+cudaError_t radix_pass_bits(const uint32_t *kin, const uint32_t *vin, uint32_t *kout,
+                            uint32_t *vout, int64_t n, int shift, const uint32_t *dig_off,
+                            unsigned long long *status, unsigned int *ctr, cudaStream_t s) {
+  const size_t smem = (size_t)NW * (1 << BITS) * 2 + (size_t)(1 << BITS) * 4;
+  static bool configured = false;
+  if (!configured) {
+    cudaFuncSetAttribute(k_radix_pass<BITS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    configured = true;
+  }
+  const int64_t tiles = (n + TILE - 1) / TILE;
+  k_radix_pass<BITS><<<(unsigned)tiles, NT, smem, s>>>(kin, vin, kout, vout, n, shift, dig_off,
+                                                       status, ctr); note_launch();
+  return cudaGetLastError();
+}
+
+cudaError_t radix_pass(int bits, const uint32_t *kin, const uint32_t *vin, uint32_t *kout,
+                       uint32_t *vout, int64_t n, int shift, const uint32_t *dig_off,
+                       unsigned long long *status, unsigned int *ctr, cudaStream_t s) {
+  switch (bits) {
+#define VPIC_RP(B) case B: return radix_pass_bits<B>(kin, vin, kout, vout, n, shift, dig_off, status, ctr, s);
+    VPIC_RP(1) VPIC_RP(2) VPIC_RP(3) VPIC_RP(4) VPIC_RP(5) VPIC_RP(6) VPIC_RP(7)
+    VPIC_RP(8) VPIC_RP(9) VPIC_RP(10) VPIC_RP(11) VPIC_RP(12) VPIC_RP(13)
+#undef VPIC_RP
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+unsigned grid_cap(int64_t n, int threads, int num_sms, int per_sm) {
+  int64_t b = (n + threads - 1) / threads;
+  const int64_t cap = (int64_t)num_sms * per_sm;
+  if (b > cap) b = cap;
+  if (b < 1) b = 1;
+  return (unsigned)b;
+}
+
+#define CK(x) do { cudaError_t e_ = (x); if (e_ != cudaSuccess) return e_; } while (0)
+
+// Run the LSD passes of `pd` over (keys0, vals0 [nullable = iota]).  Returns
+// pointers to the final keys / vals (inside the workspace).
+cudaError_t lsd_sort(const PassDesc &pd, int64_t n, uint32_t *kA, uint32_t *kB, uint32_t *vA,
+                     uint32_t *vB, const uint32_t *vals0, uint32_t *ghist, uint32_t *goff,
+                     unsigned long long *status, unsigned int *ctr, bool need_keys_out,
+                     uint32_t **k_final, uint32_t **v_final, cudaStream_t s) {
+  CK(cudaMemsetAsync(ctr, 0, 4 * MAX_PASSES, s));
+  k_scan_hist<<<pd.npass, 256, 0, s>>>(ghist, goff, pd); note_launch();
+  CK(cudaGetLastError());
+  const int64_t tiles = (n + TILE - 1) / TILE;
+  uint32_t *kin = kA, *kout = kB;
+  const uint32_t *vin = vals0;
+  uint32_t *vout = (vals0 == vA) ? vB : vA;
+  for (int q = 0; q < pd.npass; ++q) {
+    CK(cudaMemsetAsync(status, 0, 8 * (size_t)tiles * (1 << pd.bits[q]), s));
+    const bool last = q == pd.npass - 1;
+    CK(radix_pass(pd.bits[q], kin, vin, (last && !need_keys_out) ? nullptr : kout, vout, n,
+                  pd.shift[q], goff + q * (1 << MAX_BITS), status, ctr + q, s));
+    *k_final = kout;
+    *v_final = vout;
+    std::swap(kin, kout);
+    vin = vout;
+    vout = (vout == vA) ? vB : vA;
+  }
+  return cudaSuccess;
+}
+
+}  // namespace
+
+size_t sort_workspace_bytes(const vpic_ctx *c, int64_t np, int order) {
+  (void)order;
+  return layout(np, c->gk.nv).total;
+}
+
+cudaError_t launch_sort(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_t *p_out,
+                        int64_t np, int order, int64_t tile_sz, void *ws, size_t ws_bytes,
+                        int32_t *voxel_counts, int64_t *new_keys, int64_t *perm, cudaStream_t s) {
+  const int64_t nv = c->gk.nv;
+  const int sms = c->num_sms;
+  if (np == 0) {
+    if (voxel_counts) CK(cudaMemsetAsync(voxel_counts, 0, 4 * (size_t)nv, s));
+    return cudaSuccess;
+  }
+  if (order == VPIC_SORT_NONE) {
+    CK(cudaMemcpyAsync(p_out, p_in, 32 * (size_t)np, cudaMemcpyDeviceToDevice, s));
+    if (voxel_counts) CK(cudaMemsetAsync(voxel_counts, 0, 4 * (size_t)nv, s));
+    if (voxel_counts || new_keys) {
+      k_hist_voxels<<<grid_cap(np, 256, sms, 8), 256, 0, s>>>(p_in, np, voxel_counts, new_keys); note_launch();
+      CK(cudaGetLastError());
+    }
+    if (perm) {
+      k_iota64<<<grid_cap(np, 256, sms, 8), 256, 0, s>>>(perm, np); note_launch();
+      CK(cudaGetLastError());
+    }
+    return cudaSuccess;
+  }
+  const WsLayout L = layout(np, nv);
+  if (ws_bytes < L.total) return cudaErrorInvalidValue;
+  char *w = static_cast<char *>(ws);
+  uint32_t *kA = reinterpret_cast<uint32_t *>(w + L.keysA);
+  uint32_t *kB = reinterpret_cast<uint32_t *>(w + L.keysB);
+  uint32_t *vA = reinterpret_cast<uint32_t *>(w + L.valsA);
+  uint32_t *vB = reinterpret_cast<uint32_t *>(w + L.valsB);
+  uint32_t *offs = reinterpret_cast<uint32_t *>(w + L.offs);
+  uint32_t *ghist = reinterpret_cast<uint32_t *>(w + L.ghist);
+  uint32_t *goff = reinterpret_cast<uint32_t *>(w + L.goff);
+  unsigned long long *status = reinterpret_cast<unsigned long long *>(w + L.status);
+  unsigned int *ctr = reinterpret_cast<unsigned int *>(w + L.ctr);
+  unsigned int *misc = reinterpret_cast<unsigned int *>(w + L.misc);
+
+  // ---- standard order: stable LSD radix sort by voxel
+  const PassDesc pd = make_passes(bits_for((uint64_t)(nv - 1)));
+  CK(cudaMemsetAsync(ghist, 0, 4 * (size_t)MAX_PASSES * (1 << MAX_BITS), s));
+  {
+    int tot = 0;
+    for (int q = 0; q < pd.npass; ++q) tot += 1 << pd.bits[q];
+    const size_t smem = 4 * (size_t)tot;
+    static bool configured = false;
+    if (!configured) {
+      cudaFuncSetAttribute(k_keys_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, 4 * 3 * 8192);
+      configured = true;
+    }
+    k_keys_hist<<<grid_cap(np, 256, sms, 2), 256, smem, s>>>(
+        p_in, np, kA, pd, ghist, (order == VPIC_SORT_STANDARD) ? new_keys : nullptr); note_launch();
+    CK(cudaGetLastError());
+  }
+  uint32_t *K = nullptr, *P = nullptr;
+  const bool need_offs = (order != VPIC_SORT_STANDARD) || voxel_counts;
+  CK(lsd_sort(pd, np, kA, kB, vA, vB, nullptr, ghist, goff, status, ctr, need_offs, &K, &P, s));
+
+  if (need_offs) {
+    k_offsets<<<grid_cap(np, 256, sms, 16), 256, 0, s>>>(K, np, nv, offs); note_launch();
+    CK(cudaGetLastError());
+    CK(cudaMemsetAsync(misc, 0, 64, s));
+    k_counts<<<grid_cap(nv, 256, sms, 16), 256, 0, s>>>(offs, nv, voxel_counts, misc); note_launch();
+    CK(cudaGetLastError());
+  }
+  if (order == VPIC_SORT_STRIDED || order == VPIC_SORT_TILED_STRIDED) {
+    // host needs max_r, min_k and max_k to size the rank pass (one sync)
+    uint32_t h[3];
+    CK(cudaMemcpyAsync(&h[0], misc, 4, cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(&h[1], K, 4, cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(&h[2], K + np - 1, 4, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    const uint32_t max_r = h[0];
+    const int64_t min_k = h[1], max_k = h[2];
+    const int64_t T = tile_sz > 0 ? tile_sz : c->tile_sz;
+    uint64_t max_ck;
+    if (order == VPIC_SORT_STRIDED) max_ck = max_r ? max_r - 1 : 0;
+    else max_ck = (uint64_t)(max_k / T - min_k / T) * max_r + (max_r ? max_r - 1 : 0);
+    if (max_ck >> 32) return cudaErrorInvalidValue;  // composite key beyond 32 bits
+    const PassDesc pr = make_passes(bits_for(max_ck));
+    // the standard keys/perm live in (K, P); use the other buffers for the rank pass
+    uint32_t *ck = (K == kA) ? kB : kA;
+    uint32_t *vfree = (P == vA) ? vB : vA;
+    CK(cudaMemsetAsync(ghist, 0, 4 * (size_t)MAX_PASSES * (1 << MAX_BITS), s));
+    {
+      int tot = 0;
+      for (int q = 0; q < pr.npass; ++q) tot += 1 << pr.bits[q];
+      static bool configured = false;
+      if (!configured) {
+        cudaFuncSetAttribute(k_rank_keys, cudaFuncAttributeMaxDynamicSharedMemorySize, 4 * 3 * 8192);
+        configured = true;
+      }
+      k_rank_keys<<<grid_cap(np, 256, sms, 2), 256, 4 * (size_t)tot, s>>>(
+          K, P, offs, np, order, T, max_r, ck, pr, ghist, new_keys); note_launch();
+      CK(cudaGetLastError());
+    }
+    // the rank pass permutes the standard perm P; K (standard keys) is free now
+    // buffers: keys ck -> other = K ; vals P -> vfree
+    uint32_t *kX = ck, *kY = K, *vX = P, *vY = vfree;
+    uint32_t *K2 = nullptr, *P2 = nullptr;
+    CK(lsd_sort(pr, np, kX, kY, vX, vY, P, ghist, goff, status, ctr, false, &K2, &P2, s));
+    P = P2;
+  }
+  k_gather<<<grid_cap(np, 256, sms, 16), 256, 0, s>>>(p_in, p_out, P, np, perm); note_launch();
+  return cudaGetLastError();
+}
+
+}  // namespace vpic

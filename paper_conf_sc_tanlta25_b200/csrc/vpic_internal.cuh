@@ -1,0 +1,97 @@
+// Internal declarations shared by the libvpic.so translation units.
+// Nothing here is shared with oracle/ (the two are independent by design).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/vpic.h"
+
+namespace vpic {
+
+// Grid constants passed by value to kernels (kernel-param constant bank).
+struct GridK {
+  int32_t nx, ny, nz;
+  int32_t sx, sy;            // nx+2, ny+2
+  int32_t sxy;               // sx*sy
+  int64_t nv;
+  float cdt_dx, cdt_dy, cdt_dz;
+  float dt, cvac;
+  // per face: 0 = local neighbour/wrap, 1 = reflect, 2 = absorb, 3 = remote
+  int32_t face_kind[6];
+};
+
+enum FaceKind { FACE_LOCAL = 0, FACE_REFLECT = 1, FACE_ABSORB = 2, FACE_REMOTE = 3 };
+
+enum MathMode { MATH_FAST = 0, MATH_IEEE = 1 };
+enum DepositMode { DEP_AUTO = 0, DEP_LANE = 1, DEP_WARP = 2 };
+enum AdvanceKernel { ADV_AUTO = 0, ADV_DIRECT = 1, ADV_TMA = 2 };
+
+struct Exchange;  // multi-GPU state (migrate.cu)
+
+}  // namespace vpic
+
+struct vpic_ctx {
+  vpic_grid_t g;
+  vpic::GridK gk;
+  int rank, nranks, device;
+  int num_sms;
+  int64_t l2_bytes;
+  int64_t tile_sz;
+  int math, deposit, adv_kernel;
+  bool periodic_local[3];  // axis wraps locally (both faces local periodic)
+  vpic::Exchange *ex;      // null when nranks == 1
+  // small device scratch owned by the context
+  void *scratch;
+  size_t scratch_bytes;
+  int64_t *d_count;        // device counters [4]
+};
+
+namespace vpic {
+
+// process-wide count of kernels launched by the library (vpic_kernel_launches)
+void note_launch(int n = 1);
+
+// ---- launchers implemented in the .cu files (return cudaError_t) ----------
+cudaError_t launch_advance_p(const vpic_ctx *c, float qsp, float msp, vpic_particle_t *p,
+                             int64_t np, const float *interp, float *acc, vpic_mover_t *movers,
+                             int64_t max_movers, int64_t *n_movers, int32_t *flags,
+                             cudaStream_t s);
+// the two math variants are compiled from the same source (advance_p.cu)
+cudaError_t launch_advance_p_fast(const vpic_ctx *c, float qsp, float msp, vpic_particle_t *p,
+                                  int64_t np, const float *interp, float *acc,
+                                  vpic_mover_t *movers, int64_t max_movers, int64_t *n_movers,
+                                  int32_t *flags, cudaStream_t s);
+cudaError_t launch_advance_p_ieee(const vpic_ctx *c, float qsp, float msp, vpic_particle_t *p,
+                                  int64_t np, const float *interp, float *acc,
+                                  vpic_mover_t *movers, int64_t max_movers, int64_t *n_movers,
+                                  int32_t *flags, cudaStream_t s);
+// move_p of a list of movers (incoming particles after migration)
+cudaError_t launch_move_movers_fast(const vpic_ctx *c, float qsp, vpic_particle_t *p,
+                                    const vpic_mover_t *in, int64_t n_in, float *acc,
+                                    vpic_mover_t *out, int64_t max_out, int64_t *n_out,
+                                    int32_t *flags, cudaStream_t s);
+cudaError_t launch_move_movers_ieee(const vpic_ctx *c, float qsp, vpic_particle_t *p,
+                                    const vpic_mover_t *in, int64_t n_in, float *acc,
+                                    vpic_mover_t *out, int64_t max_out, int64_t *n_out,
+                                    int32_t *flags, cudaStream_t s);
+
+cudaError_t launch_fill_ghosts(const vpic_ctx *c, float *fields, cudaStream_t s);
+cudaError_t launch_load_interp(const vpic_ctx *c, const float *fields, float *interp,
+                               cudaStream_t s);
+cudaError_t launch_unload(const vpic_ctx *c, const float *acc, float *jf, cudaStream_t s);
+
+size_t sort_workspace_bytes(const vpic_ctx *c, int64_t np, int order);
+cudaError_t launch_sort(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_t *p_out,
+                        int64_t np, int order, int64_t tile_sz, void *ws, size_t ws_bytes,
+                        int32_t *voxel_counts, int64_t *new_keys, int64_t *perm,
+                        cudaStream_t s);
+
+int migrate(vpic_ctx *c, float qsp, float msp, vpic_particle_t *p, int64_t *np, int64_t max_np,
+            vpic_mover_t *movers, const int64_t *n_movers, float *acc, cudaStream_t s);
+int exchange_create(vpic_ctx *c, const uint8_t *uid);
+void exchange_destroy(vpic_ctx *c);
+int halo_fields(vpic_ctx *c, float *fields, cudaStream_t s);
+int reduce_jf(vpic_ctx *c, float *jf, cudaStream_t s);
+
+}  // namespace vpic

@@ -260,3 +260,36 @@ def random_particles(g: GridSpec, n: int, seed: int, u_scale: float = 0.5,
         p[k] = rng.standard_normal(n, dtype=np.float32) * np.float32(u_scale)
     p["w"] = rng.random(n, dtype=np.float32) + np.float32(0.5)
     return p
+
+
+# ------------------------------------------------------- decomposition --
+PROCESS_GRIDS = {1: (1, 1, 1), 2: (2, 1, 1), 4: (2, 2, 1), 8: (2, 2, 2)}
+
+
+def process_grid(nranks: int) -> Tuple[int, int, int]:
+    if nranks in PROCESS_GRIDS:
+        return PROCESS_GRIDS[nranks]
+    return (nranks, 1, 1)
+
+
+def decompose(block: GridSpec, nranks: int, rank: int) -> GridSpec:
+    """Rank `rank`'s block of a periodic box tiled by `block`-sized blocks on
+    the process grid of `nranks` (x fastest).  PERIODIC faces point at the
+    neighbour rank (a local wrap when the process grid is 1 wide there)."""
+    P = process_grid(nranks)
+    c = (rank % P[0], (rank // P[0]) % P[1], rank // (P[0] * P[1]))
+
+    def rank_of(cc):
+        cc = [cc[a] % P[a] for a in range(3)]
+        return cc[0] + P[0] * (cc[1] + P[1] * cc[2])
+
+    nbr = []
+    for f in range(6):
+        a = f % 3
+        d = -1 if f < 3 else 1
+        cc = list(c)
+        cc[a] += d
+        nbr.append(rank_of(cc))
+    n = (block.nx, block.ny, block.nz)
+    return replace(block, nbr_rank=tuple(nbr), rank=rank,
+                   gx0=c[0] * n[0], gy0=c[1] * n[1], gz0=c[2] * n[2])

@@ -1,0 +1,122 @@
+"""The hot path as a user drives it: device-resident state for one rank and a
+PIC step made only of libvpic C-ABI calls:
+
+    [every S steps] vpic_sort_particles (per species)
+    vpic_load_interpolator -> vpic_clear_accumulator
+    -> vpic_advance_p (per species) -> [vpic_migrate_particles]
+    -> vpic_unload_accumulator
+
+PyTorch only provides device memory, pinned host memory and the stream.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+from typing import List, Optional
+
+import numpy as np
+import torch
+
+from . import inputs, vpic
+
+
+@dataclass
+class SpeciesState:
+    name: str
+    q: float
+    m: float
+    p: torch.Tensor          # [cap, 8] float32 (32-B records)
+    scratch: torch.Tensor    # sort output buffer, same shape
+    np: int
+    movers: torch.Tensor     # [max_movers, 4]
+    n_movers: torch.Tensor   # int64[1]
+    flags: torch.Tensor      # int32[1]
+
+
+class HotPath:
+    def __init__(self, wl: inputs.Workload, species_particles: List[np.ndarray], fields: np.ndarray,
+                 order: int = vpic.VPIC_SORT_STANDARD, math: int = vpic.MATH_FAST,
+                 deposit: int = vpic.DEP_AUTO, tile_sz: int = 0, rank: int = 0, nranks: int = 1,
+                 uid: bytes = None, capacity_factor: float = 1.0, max_movers: int = 1 << 20,
+                 device: Optional[int] = None):
+        vpic.load()
+        self.wl = wl
+        self.g = wl.grid
+        self.dev = torch.device("cuda", torch.cuda.current_device() if device is None else device)
+        self.ctx = vpic.Context(self.g, rank, nranks, uid, self.dev.index)
+        self.ctx.set_option(vpic.VPIC_OPT_MATH, math)
+        self.ctx.set_option(vpic.VPIC_OPT_DEPOSIT, deposit)
+        self.order = order
+        self.tile_sz = tile_sz
+        self.nranks = nranks
+        self.migrate = nranks > 1 or any(b == inputs.BC_ABSORB for b in self.g.pbc)
+        nv = self.g.nv
+        f32 = dict(dtype=torch.float32, device=self.dev)
+        self.fields = torch.from_numpy(np.ascontiguousarray(fields)).to(self.dev)
+        self.interp = torch.zeros((nv, 20), **f32)
+        self.acc = torch.zeros((nv, 12), **f32)
+        self.jf = torch.zeros((nv, 4), **f32)
+        self.species: List[SpeciesState] = []
+        max_np = 0
+        for sp, ph in zip(wl.species, species_particles):
+            n = int(ph.size)
+            cap = max(1, int(n * capacity_factor))
+            p = torch.empty((cap, 8), **f32)
+            if n:
+                p[:n].copy_(torch.from_numpy(np.ascontiguousarray(ph).view(np.float32).reshape(-1, 8)))
+            self.species.append(SpeciesState(
+                sp.name, sp.q, sp.m, p, torch.empty_like(p), n,
+                torch.zeros((max_movers, 4), **f32),
+                torch.zeros(1, dtype=torch.int64, device=self.dev),
+                torch.zeros(1, dtype=torch.int32, device=self.dev)))
+            max_np = max(max_np, cap)
+        ws = vpic.vpic_sort_workspace_bytes(self.ctx, max_np, order)
+        self.ws = torch.empty(max(ws, 1), dtype=torch.uint8, device=self.dev)
+        self.adv_events = []   # (start, end) CUDA events around advance_p, when recording
+        self.record_advance = False
+
+    # ------------------------------------------------------------ calls --
+    @property
+    def n_particles(self) -> int:
+        return sum(s.np for s in self.species)
+
+    def sort(self, order: Optional[int] = None):
+        order = self.order if order is None else order
+        if order == vpic.VPIC_SORT_NONE:
+            return
+        for s in self.species:
+            vpic.vpic_sort_particles(self.ctx, s.p, s.scratch, s.np, order, self.tile_sz, self.ws)
+            s.p, s.scratch = s.scratch, s.p
+
+    def step(self, do_sort: bool = False):
+        if do_sort:
+            self.sort()
+        vpic.vpic_load_interpolator(self.ctx, self.fields, self.interp)
+        vpic.vpic_clear_accumulator(self.ctx, self.acc)
+        stream = torch.cuda.current_stream()
+        for s in self.species:
+            if self.record_advance:
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(stream)
+            vpic.vpic_advance_p(self.ctx, s.q, s.m, s.p, s.np, self.interp, self.acc, s.movers,
+                                s.movers.shape[0], s.n_movers, s.flags)
+            if self.record_advance:
+                e1.record(stream)
+                self.adv_events.append((e0, e1, s.np))
+            if self.migrate:
+                s.np = vpic.vpic_migrate_particles(self.ctx, s.q, s.m, s.p, s.np, s.p.shape[0],
+                                                   s.movers, s.n_movers, self.acc)
+                s.n_movers.zero_()
+        vpic.vpic_unload_accumulator(self.ctx, self.acc, self.jf)
+
+    def cycle(self, steps: int):
+        """One sort period: sort, then `steps` PIC steps."""
+        for k in range(steps):
+            self.step(do_sort=(k == 0))
+
+    # ------------------------------------------------------- host <-> device --
+    def particles_host(self, k: int) -> np.ndarray:
+        s = self.species[k]
+        return vpic.particles_to_host(s.p[:s.np])
+
+    def close(self):
+        self.ctx.close()

@@ -1,0 +1,54 @@
+"""Comparison helpers for the GPU-vs-oracle parity tests (tolerances of
+BASELINE.json north_star / SURVEY.md §8(c) c.4, restated in DESIGN.md)."""
+import numpy as np
+
+from paper_conf_sc_tanlta25_b200 import inputs
+
+ULP1 = float(np.spacing(np.float32(1.0)))   # 2^-23
+OFFSET_TOL = 4 * ULP1                       # 4 ulp(1.0) on the cell offsets
+
+
+def global_pos(g, p):
+    x, y, z = g.coords(p["i"].astype(np.int64))
+    return np.stack([x + (1 + p["dx"].astype(np.float64)) / 2,
+                     y + (1 + p["dy"].astype(np.float64)) / 2,
+                     z + (1 + p["dz"].astype(np.float64)) / 2], -1)
+
+
+def assert_particles_bitexact(a, b):
+    va = np.ascontiguousarray(a).view(np.uint32).reshape(-1, 8)
+    vb = np.ascontiguousarray(b).view(np.uint32).reshape(-1, 8)
+    bad = np.nonzero((va != vb).any(1))[0]
+    assert bad.size == 0, f"{bad.size} particles differ, first {bad[:5]}: {a[bad[:3]]} vs {b[bad[:3]]}"
+
+
+def assert_particles_close(g, gpu, orc, u_old):
+    """Per particle, in the oracle's voxel frame (a face tie may put the GPU
+    particle in the neighbouring voxel: compare global positions, periodic
+    wrap folded): |d offset| <= 4 ulp(1); |du| <= max(4 ulp(u), 1e-6 max(|u|,|u_old|))."""
+    assert gpu.shape == orc.shape
+    n = np.array([g.nx, g.ny, g.nz], np.float64)
+    d = global_pos(g, gpu) - global_pos(g, orc)
+    d = d - n * np.round(d / n)
+    off_err = 2 * np.abs(d)   # offset units: 2 per cell
+    assert off_err.max(initial=0) <= OFFSET_TOL, f"max offset err {off_err.max()}"
+    for k, c in enumerate(("ux", "uy", "uz")):
+        ug, uo = gpu[c].astype(np.float64), orc[c].astype(np.float64)
+        tol = np.maximum(4 * np.spacing(np.abs(orc[c])).astype(np.float64),
+                         1e-6 * np.maximum(np.abs(uo), np.abs(u_old[:, k])))
+        err = np.abs(ug - uo)
+        bad = np.nonzero(err > tol)[0]
+        assert bad.size == 0, f"{c}: {bad.size} out of tol, worst {err[bad].max()} vs {tol[bad].min()}"
+    assert np.array_equal(gpu["w"], orc["w"])
+
+
+def assert_acc_close(acc_gpu, acc_orc, acc_abs, rel=1e-5):
+    """|a_gpu - a_orc| <= rel * sum|contributions| per entry (atomic reordering only)."""
+    err = np.abs(acc_gpu.astype(np.float64) - acc_orc.astype(np.float64))
+    tol = rel * acc_abs + 1e-30
+    bad = np.argwhere(err > tol)
+    assert bad.size == 0, f"{len(bad)} acc entries out of tol; worst err {err.max()}, at {bad[:3]}"
+
+
+def u_of(p):
+    return np.stack([p["ux"], p["uy"], p["uz"]], 1).astype(np.float64)

@@ -1,0 +1,267 @@
+"""GPU parity: every C-ABI call against the oracle on identical seeded inputs.
+
+Bars: sort keys, counts, new keys and permutation
+bit-exact; interpolator bit-exact; particles bit-exact in IEEE mode and within
+4 ulp / 1e-6 (oracle voxel frame) in FAST mode; accumulators and jf within
+1e-5 of the sum of absolute contributions (atomic reordering only).
+"""
+import numpy as np
+import pytest
+import torch
+
+from paper_conf_sc_tanlta25_b200 import inputs
+from parity_util import (assert_acc_close, assert_particles_bitexact, assert_particles_close,
+                         u_of)
+
+pytestmark = pytest.mark.gpu
+PD = inputs.PARTICLE_DTYPE
+
+
+@pytest.fixture(scope="module")
+def V():
+    from paper_conf_sc_tanlta25_b200 import _build, vpic
+    _build.build()
+    vpic.load()
+    assert torch.cuda.is_available(), "gpu tests need a B200"
+    return vpic
+
+
+def mkctx(V, g, math=0, deposit=0):
+    c = V.Context(g)
+    c.set_option(V.VPIC_OPT_MATH, math)
+    c.set_option(V.VPIC_OPT_DEPOSIT, deposit)
+    return c
+
+
+def dev_particles(V, p):
+    return V.particles_to_device(p)
+
+
+# ------------------------------------------------------------------ sort --
+def sort_cases():
+    out = []
+    wl = inputs.config(0)
+    pe = inputs.make_species_particles(wl)[0]
+    out.append(("c1_sorted", wl.grid, pe))
+    out.append(("c1_shuffled", wl.grid, inputs.shuffle(pe, 1)))
+    g = inputs.GridSpec(7, 5, 3)
+    out.append(("random_ragged", g, inputs.random_particles(g, 8193, 2)))
+    out.append(("three_voxels", g, inputs.random_particles(g, 5000, 3, vox=[g.voxel(1, 1, 1), g.voxel(7, 5, 3), g.voxel(3, 2, 2)])))
+    out.append(("one_voxel", g, inputs.random_particles(g, 10000, 4, vox=[g.voxel(4, 3, 2)])))
+    out.append(("single", g, inputs.random_particles(g, 1, 5)))
+    out.append(("warp_minus_one", g, inputs.random_particles(g, 31, 6)))
+    g2 = inputs.GridSpec(32, 32, 32)
+    out.append(("many_tiles", g2, inputs.shuffle(inputs.random_particles(g2, 200000, 7), 8)))
+    return out
+
+
+@pytest.mark.parametrize("case", sort_cases(), ids=lambda c: c[0])
+@pytest.mark.parametrize("order,T", [(0, 0), (1, 0), (2, 7), (2, 1), (2, 0), (3, 0)])
+def test_sort_parity(V, orc, case, order, T):
+    name, g, p = case
+    ctx = mkctx(V, g)
+    Tq = T if T else ctx.info()["tile_sz"]
+    p_out_o, counts_o, nk_o, perm_o = orc.sort_particles(g, p, order, Tq)
+    n = p.size
+    p_in = dev_particles(V, p)
+    p_out = torch.empty_like(p_in)
+    ws = torch.empty(V.vpic_sort_workspace_bytes(ctx, n, order), dtype=torch.uint8, device="cuda")
+    counts = torch.full((g.nv,), -7, dtype=torch.int32, device="cuda")
+    nk = torch.empty(n, dtype=torch.int64, device="cuda")
+    perm = torch.empty(n, dtype=torch.int64, device="cuda")
+    V.vpic_sort_particles(ctx, p_in, p_out, n, order, T, ws, counts, nk, perm)
+    torch.cuda.synchronize()
+    assert_particles_bitexact(V.particles_to_host(p_out), p_out_o)
+    assert np.array_equal(counts.cpu().numpy(), counts_o)
+    assert np.array_equal(perm.cpu().numpy(), perm_o)
+    assert np.array_equal(nk.cpu().numpy(), nk_o)
+    # input untouched
+    assert_particles_bitexact(V.particles_to_host(p_in), p)
+
+
+def test_sort_three_passes(V, orc):
+    """nv > 2^26: the standard sort needs three <= 13-bit digit passes."""
+    g = inputs.GridSpec(512, 512, 256)
+    p = inputs.random_particles(g, 100000, 9)
+    ctx = mkctx(V, g)
+    p_out_o, counts_o, _, perm_o = orc.sort_particles(g, p, 0)
+    p_in = dev_particles(V, p)
+    p_out = torch.empty_like(p_in)
+    ws = torch.empty(V.vpic_sort_workspace_bytes(ctx, p.size, 0), dtype=torch.uint8, device="cuda")
+    counts = torch.empty(g.nv, dtype=torch.int32, device="cuda")
+    perm = torch.empty(p.size, dtype=torch.int64, device="cuda")
+    V.vpic_sort_particles(ctx, p_in, p_out, p.size, 0, 0, ws, counts, None, perm)
+    assert np.array_equal(perm.cpu().numpy(), perm_o)
+    assert np.array_equal(counts.cpu().numpy(), counts_o)
+
+
+def test_sort_empty(V):
+    g = inputs.GridSpec(4, 4, 4)
+    ctx = mkctx(V, g)
+    counts = torch.full((g.nv,), 5, dtype=torch.int32, device="cuda")
+    x = torch.empty((0, 8), device="cuda")
+    for order in range(4):
+        V.vpic_sort_particles(ctx, x, torch.empty_like(x), 0, order, 0, None, counts)
+        assert int(counts.abs().sum()) == 0
+
+
+# ----------------------------------------------------- interp / advance --
+def adv_cases():
+    wl = inputs.config(0)
+    ps = inputs.make_species_particles(wl)
+    g = wl.grid
+    f = inputs.make_fields(g, 0.01)
+    out = [("c1_electrons", g, ps[0], -1.0, 1.0, f), ("c1_ions", g, ps[1], 1.0, 25.0, f)]
+    gh = inputs.GridSpec(9, 6, 5, pbc=(0, 0, 1, 0, 0, 1))
+    out.append(("reflect_z_hot", gh, inputs.random_particles(gh, 20000, 11, u_scale=1.0), -1.0, 1.0,
+                inputs.make_fields(gh, 0.05, seed=3)))
+    gr = inputs.GridSpec(5, 6, 7)
+    out.append(("periodic_hot_ragged", gr, inputs.random_particles(gr, 12345, 12, u_scale=1.2), 0.7,
+                1.3, inputs.make_fields(gr, 0.2, seed=4)))
+    return out
+
+
+def run_both(V, orc, g, p, q, m, fields, math, deposit):
+    interp_o = orc.load_interpolator(g, fields.copy())
+    acc_o = np.zeros((g.nv, 12), np.float32)
+    acc_abs = np.zeros((g.nv, 12), np.float64)
+    p_o = p.copy()
+    mv_o = orc.advance_p(g, q, m, p_o, interp_o, acc_o, acc_abs)
+    ctx = mkctx(V, g, math, deposit)
+    fd = torch.from_numpy(fields.copy()).cuda()
+    interp = torch.zeros((g.nv, 20), dtype=torch.float32, device="cuda")
+    V.vpic_load_interpolator(ctx, fd, interp)
+    acc = torch.empty((g.nv, 12), dtype=torch.float32, device="cuda")
+    V.vpic_clear_accumulator(ctx, acc)
+    pd = dev_particles(V, p)
+    movers = torch.zeros((max(p.size, 1), 4), dtype=torch.float32, device="cuda")
+    nm = torch.zeros(1, dtype=torch.int64, device="cuda")
+    flags = torch.zeros(1, dtype=torch.int32, device="cuda")
+    V.vpic_advance_p(ctx, q, m, pd, p.size, interp, acc, movers, p.size, nm, flags)
+    torch.cuda.synchronize()
+    return dict(interp_o=interp_o, acc_o=acc_o, acc_abs=acc_abs, p_o=p_o, mv_o=mv_o,
+                interp=interp.cpu().numpy(), acc=acc.cpu().numpy(), p=V.particles_to_host(pd),
+                nm=int(nm.item()), flags=int(flags.item()), ctx=ctx, fields=fd.cpu().numpy(),
+                acc_t=acc)
+
+
+@pytest.mark.parametrize("case", adv_cases(), ids=lambda c: c[0])
+@pytest.mark.parametrize("deposit", [1, 2])
+def test_advance_ieee_bitexact(V, orc, case, deposit):
+    name, g, p, q, m, f = case
+    r = run_both(V, orc, g, p, q, m, f, V.MATH_IEEE, deposit)
+    vox = g.interior_voxels()
+    assert np.array_equal(r["interp"][vox], r["interp_o"][vox])
+    assert_particles_bitexact(r["p"], r["p_o"])
+    assert_acc_close(r["acc"], r["acc_o"], r["acc_abs"])
+    assert r["nm"] == 0 and r["flags"] == 0
+
+
+@pytest.mark.parametrize("case", adv_cases(), ids=lambda c: c[0])
+@pytest.mark.parametrize("deposit", [1, 2])
+def test_advance_fast_tolerance(V, orc, case, deposit):
+    name, g, p, q, m, f = case
+    r = run_both(V, orc, g, p, q, m, f, V.MATH_FAST, deposit)
+    assert_particles_close(g, r["p"], r["p_o"], u_of(p))
+    assert_acc_close(r["acc"], r["acc_o"], r["acc_abs"])
+
+
+def test_ghost_fill_matches(V, orc):
+    g = inputs.GridSpec(6, 5, 4)
+    f = inputs.make_fields(g, 1.0, seed=9)
+    r = run_both(V, orc, g, inputs.random_particles(g, 10, 1), 1.0, 1.0, f, V.MATH_IEEE, 1)
+    fo = f.copy()
+    orc.load_interpolator(g, fo)
+    assert np.array_equal(r["fields"], fo)
+
+
+@pytest.mark.parametrize("case", adv_cases()[2:], ids=lambda c: c[0])
+def test_unload_parity(V, orc, case):
+    name, g, p, q, m, f = case
+    r = run_both(V, orc, g, p, q, m, f, V.MATH_FAST, 2)
+    jf = torch.empty((g.nv, 4), dtype=torch.float32, device="cuda")
+    V.vpic_unload_accumulator(r["ctx"], r["acc_t"], jf)
+    jf_o = orc.unload_accumulator(g, r["acc"])
+    jf_abs = orc.unload_accumulator(g, np.abs(r["acc"])).astype(np.float64)
+    assert_acc_close(jf.cpu().numpy(), jf_o, jf_abs + 1e-30)
+
+
+def test_continuity_on_gpu_output(V, orc):
+    """Discrete continuity 4 dR + div J = 0 evaluated on the GPU's particles and
+    accumulator (FAST mode, warp deposit)."""
+    g = inputs.GridSpec(8, 8, 8, dt=0.5)
+    p = inputs.random_particles(g, 50000, 21, u_scale=0.8)
+    q = 0.7
+    rho0 = orc.accumulate_rho(g, p, q)
+    r = run_both(V, orc, g, p, q, 1.0, inputs.make_fields(g, 0.05), V.MATH_FAST, 2)
+    rho1 = orc.accumulate_rho(g, r["p"], q)
+    J = orc.unload_raw(g, r["acc"])
+    S = (g.nx + 2, g.ny + 2, g.nz + 2)
+    Jg = J[:, :3].reshape(S[2], S[1], S[0], 3).transpose(2, 1, 0, 3).copy()
+    R = (rho1 - rho0).reshape(S[2], S[1], S[0]).transpose(2, 1, 0).copy()
+    for a in range(3):
+        hi = [slice(None)] * 3; hi[a] = S[a] - 1
+        lo = [slice(None)] * 3; lo[a] = 1
+        Jg[tuple(lo)] += Jg[tuple(hi)]
+        R[tuple(lo)] += R[tuple(hi)]
+    core = (slice(1, S[0] - 1), slice(1, S[1] - 1), slice(1, S[2] - 1))
+    res = 4 * R[core]
+    for a in range(3):
+        Ja = Jg[core + (a,)]
+        res = res + Ja - np.roll(Ja, 1, axis=a)
+    scale = np.abs(4 * R[core]).max()
+    assert scale > 1
+    assert np.abs(res).max() < 2e-5 * scale
+
+
+def test_absorb_movers_and_migrate(V, orc):
+    """Absorbing z walls: movers reported, particles removed (multiset equal
+    to the oracle's back-fill; IEEE mode so records are bit-identical)."""
+    g = inputs.GridSpec(6, 6, 3, pbc=(0, 0, 2, 0, 0, 2))
+    p = inputs.random_particles(g, 9000, 31, u_scale=1.5)
+    r = run_both(V, orc, g, p, -1.0, 1.0, inputs.make_fields(g, 0.01), V.MATH_IEEE, 2)
+    assert r["nm"] == r["mv_o"].size > 0
+    assert_particles_bitexact(r["p"], r["p_o"])
+    # migrate on the GPU
+    pd = dev_particles(V, r["p"])
+    ctx = r["ctx"]
+    # rebuild the mover list on the device from the oracle's (same set)
+    movers = torch.from_numpy(r["mv_o"].copy().view(np.float32).reshape(-1, 4)).cuda()
+    nm = torch.tensor([r["mv_o"].size], dtype=torch.int64, device="cuda")
+    n_new = V.vpic_migrate_particles(ctx, -1.0, 1.0, pd, p.size, p.size, movers, nm, r["acc_t"])
+    p_left_o = orc.remove_absorbed(g, r["p_o"].copy(), r["mv_o"])
+    assert n_new == p_left_o.size
+    got = V.particles_to_host(pd[:n_new])
+    key = lambda a: np.sort(np.ascontiguousarray(a).view(np.dtype((np.void, 32))))
+    assert np.array_equal(key(got), key(p_left_o))
+
+
+def test_mover_overflow_flag(V, orc):
+    g = inputs.GridSpec(6, 6, 3, pbc=(0, 0, 2, 0, 0, 2))
+    p = inputs.random_particles(g, 9000, 31, u_scale=1.5)
+    ctx = mkctx(V, g)
+    fd = torch.from_numpy(inputs.make_fields(g, 0.01)).cuda()
+    interp = torch.zeros((g.nv, 20), device="cuda")
+    V.vpic_load_interpolator(ctx, fd, interp)
+    acc = torch.zeros((g.nv, 12), device="cuda")
+    pd = dev_particles(V, p)
+    movers = torch.zeros((4, 4), device="cuda")
+    nm = torch.zeros(1, dtype=torch.int64, device="cuda")
+    flags = torch.zeros(1, dtype=torch.int32, device="cuda")
+    V.vpic_advance_p(ctx, -1.0, 1.0, pd, p.size, interp, acc, movers, 4, nm, flags)
+    torch.cuda.synchronize()
+    assert int(nm.item()) > 4 and int(flags.item()) & 1
+
+
+def test_invalid_arguments(V):
+    g = inputs.GridSpec(4, 4, 4)
+    ctx = mkctx(V, g)
+    with pytest.raises(V.VpicError):
+        ctx.set_option(V.VPIC_OPT_MATH, 7)
+    x = torch.zeros((10, 8), device="cuda")
+    with pytest.raises(V.VpicError):  # in-place sort is rejected
+        V.vpic_sort_particles(ctx, x, x, 10, 0, 0, torch.empty(1 << 20, dtype=torch.uint8, device="cuda"))
+    with pytest.raises(V.VpicError):  # workspace too small
+        V.vpic_sort_particles(ctx, x, torch.empty_like(x), 10, 0, 0, torch.empty(16, dtype=torch.uint8, device="cuda"))
+    with pytest.raises(V.VpicError):
+        V.Context(inputs.GridSpec(4, 4, 4, nbr_rank=(1, 0, 0, 0, 0, 0)))

@@ -48,6 +48,7 @@ def parse():
     ap.add_argument("--sort-every", type=int, default=0)
     ap.add_argument("--math", default="fast", choices=["fast", "ieee"])
     ap.add_argument("--deposit", default="auto", choices=["auto", "lane", "warp"])
+    ap.add_argument("--kernel", default="auto", choices=["auto", "direct", "tma"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no e2e/cpu legs)")
@@ -230,6 +231,7 @@ def our_arm(args, rank, world):
     cap = 1.0 if world == 1 else 1.05
     hp = HotPath(wl, parts, fields, order=order, math=math_mode, deposit=dep, rank=rank,
                  nranks=world, uid=uid, capacity_factor=cap, device=local)
+    hp.ctx.set_option(vpic.VPIC_OPT_ADVANCE_KERNEL, {"auto": 0, "direct": 1, "tma": 2}[args.kernel])
     n_local = hp.n_particles
 
     def barrier():
@@ -332,7 +334,7 @@ def our_arm(args, rank, world):
         "config": {"workload": wl.name, "cells_per_gpu": [g.nx, g.ny, g.nz], "ppc_per_species": wl.ppc,
                    "species": len(wl.species), "particles": int(ntot), "sort_every": S,
                    "order": args.order, "shuffled": bool(args.shuffle), "math": args.math,
-                   "deposit": args.deposit, "parallelism": f"domain{world}",
+                   "deposit": args.deposit, "kernel": args.kernel, "parallelism": f"domain{world}",
                    "l2": "no flush: inputs (17 GB of particles per GPU) >> 126 MB L2"},
         "per_gpu": value / world,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",

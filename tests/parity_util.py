@@ -22,10 +22,21 @@ def assert_particles_bitexact(a, b):
     assert bad.size == 0, f"{bad.size} particles differ, first {bad[:5]}: {a[bad[:3]]} vs {b[bad[:3]]}"
 
 
-def assert_particles_close(g, gpu, orc, u_old):
+def kick_bound(g, p, q, m, interp):
+    """Upper bound of |2 qdt_2mc E| at each particle (|offsets| <= 1), from the
+    interpolator coefficients of its voxel: the size of the E-kick terms that
+    are added to and cancelled against u inside the push."""
+    qdt_2mc = abs(q * g.dt / (2 * m * g.cvac))
+    f = np.abs(interp[p["i"]].astype(np.float64))
+    return 2 * qdt_2mc * np.stack([f[:, 0:4].sum(1), f[:, 4:8].sum(1), f[:, 8:12].sum(1)], 1)
+
+
+def assert_particles_close(g, gpu, orc, u_old, kick=None):
     """Per particle, in the oracle's voxel frame (a face tie may put the GPU
     particle in the neighbouring voxel: compare global positions, periodic
-    wrap folded): |d offset| <= 4 ulp(1); |du| <= max(4 ulp(u), 1e-6 max(|u|,|u_old|))."""
+    wrap folded): |d offset| <= 4 ulp(1); |du| <= max(4 ulp(u), 1e-6 max(|u|,
+    |u_old|, |2 qdt_2mc E|)) -- the last term is the size of the intermediate
+    sums when the E kick cancels u (tolerance reading T2)."""
     assert gpu.shape == orc.shape
     n = np.array([g.nx, g.ny, g.nz], np.float64)
     d = global_pos(g, gpu) - global_pos(g, orc)
@@ -34,8 +45,10 @@ def assert_particles_close(g, gpu, orc, u_old):
     assert off_err.max(initial=0) <= OFFSET_TOL, f"max offset err {off_err.max()}"
     for k, c in enumerate(("ux", "uy", "uz")):
         ug, uo = gpu[c].astype(np.float64), orc[c].astype(np.float64)
-        tol = np.maximum(4 * np.spacing(np.abs(orc[c])).astype(np.float64),
-                         1e-6 * np.maximum(np.abs(uo), np.abs(u_old[:, k])))
+        scale = np.maximum(np.abs(uo), np.abs(u_old[:, k]))
+        if kick is not None:
+            scale = np.maximum(scale, kick[:, k])
+        tol = np.maximum(4 * np.spacing(np.abs(orc[c])).astype(np.float64), 1e-6 * scale)
         err = np.abs(ug - uo)
         bad = np.nonzero(err > tol)[0]
         assert bad.size == 0, f"{c}: {bad.size} out of tol, worst {err[bad].max()} vs {tol[bad].min()}"

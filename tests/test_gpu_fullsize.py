@@ -1,0 +1,126 @@
+"""Parity at BASELINE.json's full size, in the launch configuration bench.py
+times (configs[1]: uniform 128^3, 128 ppc/species, 2 species = 2^29
+particles; FAST math, AUTO deposit, standard order).
+
+* particles: a random sample of 2^16 per species recomputed one by one by the
+  oracle from the same inputs;
+* accumulators: sampled voxels recomputed by the oracle from every particle
+  that can deposit into them (the 3x3x3 block of cells around the voxel);
+* sort (strided, tiled strided, standard) of the advanced electrons: the
+  properties that define each order uniquely at any size -- a permutation,
+  keys/counts consistent, and (k, input index) / (r, k) / (floor(k/T), r, k)
+  strictly increasing.
+"""
+import numpy as np
+import pytest
+import torch
+
+from paper_conf_sc_tanlta25_b200 import inputs
+from parity_util import assert_acc_close, assert_particles_close, kick_bound, u_of
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def state(orc):
+    from paper_conf_sc_tanlta25_b200 import _build, vpic
+    from paper_conf_sc_tanlta25_b200.pic import HotPath
+    _build.build()
+    wl = inputs.config(1)
+    g = wl.grid
+    parts = inputs.make_species_particles(wl)
+    fields = inputs.make_fields(g, wl.field_amp)
+    hp = HotPath(wl, parts, fields, order=vpic.VPIC_SORT_STANDARD, math=vpic.MATH_FAST,
+                 deposit=vpic.DEP_AUTO)
+    hp.step(do_sort=True)      # sort (identity on the cell-major quiet start) + one PIC step
+    torch.cuda.synchronize()
+    interp_o = orc.load_interpolator(g, fields.copy())
+    yield dict(wl=wl, g=g, parts=parts, fields=fields, hp=hp, interp_o=interp_o, vpic=vpic)
+    hp.close()
+
+
+def test_fullsize_particles_sampled(orc, state):
+    wl, g, hp, interp_o = state["wl"], state["g"], state["hp"], state["interp_o"]
+    rng = np.random.default_rng(1)
+    for k, sp in enumerate(wl.species):
+        p0 = state["parts"][k]
+        idx = np.sort(rng.choice(p0.size, 1 << 16, replace=False))
+        got = state["vpic"].particles_to_host(hp.species[k].p[torch.from_numpy(idx).cuda()])
+        ps = p0[idx].copy()
+        acc = np.zeros((g.nv, 12), np.float32)
+        orc.advance_p(g, sp.q, sp.m, ps, interp_o, acc)
+        assert_particles_close(g, got, ps, u_of(p0[idx]), kick_bound(g, p0[idx], sp.q, sp.m, interp_o))
+
+
+def test_fullsize_accumulator_sampled(orc, state):
+    wl, g, hp, interp_o = state["wl"], state["g"], state["hp"], state["interp_o"]
+    acc_gpu = hp.acc
+    rng = np.random.default_rng(2)
+    cells = [(1, 1, 1), (128, 128, 128), (64, 1, 128)] + [tuple(rng.integers(1, 129, 3)) for _ in range(5)]
+    ppc = wl.ppc
+    for (x, y, z) in cells:
+        acc = np.zeros((g.nv, 12), np.float32)
+        aabs = np.zeros((g.nv, 12), np.float64)
+        for k, sp in enumerate(wl.species):
+            p0 = state["parts"][k]
+            sel = []
+            for dz in (-1, 0, 1):
+                for dy in (-1, 0, 1):
+                    for dx in (-1, 0, 1):
+                        cx, cy, cz = [(c - 1 + d) % 128 for c, d in ((x, dx), (y, dy), (z, dz))]
+                        cell = cx + 128 * (cy + 128 * cz)   # quiet start: cell-major, ppc per cell
+                        sel.append(np.arange(cell * ppc, (cell + 1) * ppc))
+            ps = p0[np.concatenate(sel)].copy()
+            orc.advance_p(g, sp.q, sp.m, ps, interp_o, acc, aabs)
+        v = g.voxel(x, y, z)
+        got = acc_gpu[v].cpu().numpy()[None]
+        assert_acc_close(got, acc[v][None], aabs[v][None])
+
+
+def _ranks_from_standard(keys_std):
+    """r of each standard-order position: position minus the first position of its key."""
+    n = keys_std.numel()
+    pos = torch.arange(n, device=keys_std.device)
+    start = torch.ones(n, dtype=torch.bool, device=keys_std.device)
+    start[1:] = keys_std[1:] != keys_std[:-1]
+    first = torch.where(start, pos, torch.zeros_like(pos))
+    first = torch.cummax(first, 0).values
+    return pos - first
+
+
+@pytest.mark.parametrize("order", [1, 2, 0])
+def test_fullsize_sort_properties(state, order):
+    vpic, g, hp = state["vpic"], state["g"], state["hp"]
+    s = hp.species[0]                       # electrons after one push (no longer sorted)
+    n = s.np
+    p_in = s.p[:n]
+    keys_in = p_in[:, 3].contiguous().view(torch.int32).long()
+    out = torch.empty_like(p_in)
+    perm = torch.empty(n, dtype=torch.int64, device="cuda")
+    counts = torch.empty(g.nv, dtype=torch.int32, device="cuda")
+    T = hp.ctx.info()["tile_sz"]
+    vpic.vpic_sort_particles(hp.ctx, p_in, out, n, order, 0, hp.ws, counts, None, perm)
+    torch.cuda.synchronize()
+    # a permutation, payload moved with it, counts consistent
+    assert torch.equal(torch.sort(perm).values, torch.arange(n, device="cuda"))
+    assert torch.equal(out, p_in[perm])
+    assert torch.equal(counts.long(), torch.bincount(keys_in, minlength=g.nv))
+    k = keys_in[perm]
+    # rank of each input particle among equal keys, in input order
+    std = torch.sort(keys_in, stable=True).indices
+    r_in = torch.empty(n, dtype=torch.int64, device="cuda")
+    r_in[std] = _ranks_from_standard(keys_in[std])
+    r = r_in[perm]
+    if order == 0:
+        tup = [k, perm]
+    elif order == 1:
+        tup = [r, k]
+    else:
+        tup = [k // T, r, k]
+    # strictly increasing lexicographic tuples
+    gt = torch.zeros(n - 1, dtype=torch.bool, device="cuda")
+    eq = torch.ones(n - 1, dtype=torch.bool, device="cuda")
+    for c in tup:
+        gt |= eq & (c[1:] > c[:-1])
+        eq &= c[1:] == c[:-1]
+    assert bool(gt.all())

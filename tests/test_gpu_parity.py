@@ -11,7 +11,7 @@ import torch
 
 from paper_conf_sc_tanlta25_b200 import inputs
 from parity_util import (assert_acc_close, assert_particles_bitexact, assert_particles_close,
-                         u_of)
+                         kick_bound, u_of)
 
 pytestmark = pytest.mark.gpu
 PD = inputs.PARTICLE_DTYPE
@@ -26,10 +26,11 @@ def V():
     return vpic
 
 
-def mkctx(V, g, math=0, deposit=0):
+def mkctx(V, g, math=0, deposit=0, kernel=0):
     c = V.Context(g)
     c.set_option(V.VPIC_OPT_MATH, math)
     c.set_option(V.VPIC_OPT_DEPOSIT, deposit)
+    c.set_option(V.VPIC_OPT_ADVANCE_KERNEL, kernel)
     return c
 
 
@@ -121,13 +122,13 @@ def adv_cases():
     return out
 
 
-def run_both(V, orc, g, p, q, m, fields, math, deposit):
+def run_both(V, orc, g, p, q, m, fields, math, deposit, kernel=0):
     interp_o = orc.load_interpolator(g, fields.copy())
     acc_o = np.zeros((g.nv, 12), np.float32)
     acc_abs = np.zeros((g.nv, 12), np.float64)
     p_o = p.copy()
     mv_o = orc.advance_p(g, q, m, p_o, interp_o, acc_o, acc_abs)
-    ctx = mkctx(V, g, math, deposit)
+    ctx = mkctx(V, g, math, deposit, kernel)
     fd = torch.from_numpy(fields.copy()).cuda()
     interp = torch.zeros((g.nv, 20), dtype=torch.float32, device="cuda")
     V.vpic_load_interpolator(ctx, fd, interp)
@@ -147,9 +148,10 @@ def run_both(V, orc, g, p, q, m, fields, math, deposit):
 
 @pytest.mark.parametrize("case", adv_cases(), ids=lambda c: c[0])
 @pytest.mark.parametrize("deposit", [1, 2])
-def test_advance_ieee_bitexact(V, orc, case, deposit):
+@pytest.mark.parametrize("kernel", [1, 2], ids=["direct", "tma"])
+def test_advance_ieee_bitexact(V, orc, case, deposit, kernel):
     name, g, p, q, m, f = case
-    r = run_both(V, orc, g, p, q, m, f, V.MATH_IEEE, deposit)
+    r = run_both(V, orc, g, p, q, m, f, V.MATH_IEEE, deposit, kernel)
     vox = g.interior_voxels()
     assert np.array_equal(r["interp"][vox], r["interp_o"][vox])
     assert_particles_bitexact(r["p"], r["p_o"])
@@ -159,10 +161,11 @@ def test_advance_ieee_bitexact(V, orc, case, deposit):
 
 @pytest.mark.parametrize("case", adv_cases(), ids=lambda c: c[0])
 @pytest.mark.parametrize("deposit", [1, 2])
-def test_advance_fast_tolerance(V, orc, case, deposit):
+@pytest.mark.parametrize("kernel", [1, 2], ids=["direct", "tma"])
+def test_advance_fast_tolerance(V, orc, case, deposit, kernel):
     name, g, p, q, m, f = case
-    r = run_both(V, orc, g, p, q, m, f, V.MATH_FAST, deposit)
-    assert_particles_close(g, r["p"], r["p_o"], u_of(p))
+    r = run_both(V, orc, g, p, q, m, f, V.MATH_FAST, deposit, kernel)
+    assert_particles_close(g, r["p"], r["p_o"], u_of(p), kick_bound(g, p, q, m, r["interp_o"]))
     assert_acc_close(r["acc"], r["acc_o"], r["acc_abs"])
 
 
@@ -214,12 +217,13 @@ def test_continuity_on_gpu_output(V, orc):
     assert np.abs(res).max() < 2e-5 * scale
 
 
-def test_absorb_movers_and_migrate(V, orc):
+@pytest.mark.parametrize("kernel", [1, 2], ids=["direct", "tma"])
+def test_absorb_movers_and_migrate(V, orc, kernel):
     """Absorbing z walls: movers reported, particles removed (multiset equal
     to the oracle's back-fill; IEEE mode so records are bit-identical)."""
     g = inputs.GridSpec(6, 6, 3, pbc=(0, 0, 2, 0, 0, 2))
     p = inputs.random_particles(g, 9000, 31, u_scale=1.5)
-    r = run_both(V, orc, g, p, -1.0, 1.0, inputs.make_fields(g, 0.01), V.MATH_IEEE, 2)
+    r = run_both(V, orc, g, p, -1.0, 1.0, inputs.make_fields(g, 0.01), V.MATH_IEEE, 2, kernel)
     assert r["nm"] == r["mv_o"].size > 0
     assert_particles_bitexact(r["p"], r["p_o"])
     # migrate on the GPU

@@ -266,6 +266,9 @@ def our_arm(args, rank, world):
     ms = e0.elapsed_time(e1)
     adv = [(a.elapsed_time(b), n) for a, b, n in hp.adv_events]
     adv_ms = sum(t for t, _ in adv) / len(adv)
+    nsp = len(hp.species)
+    by_step = [round(sum(adv[(c * S + k) * nsp + j][0] for c in range(args.steps) for j in range(nsp))
+                     / (args.steps * nsp), 3) for k in range(S)]
     adv_np = sum(n for _, n in adv) / len(adv)
     t = torch.tensor([ms, float(pushes_local), float(n_local)], dtype=torch.float64, device=dev)
     if world > 1:
@@ -341,7 +344,8 @@ def our_arm(args, rank, world):
                      "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
                      "kernel": "k_advance (advance_p, one species per launch)",
                      "alg_bytes_per_launch": alg_bytes, "avg_launch_ms": adv_ms,
-                     "share_of_step": adv_share, "frac_of_8TBs": achieved / 8000.0},
+                     "share_of_step": adv_share, "frac_of_8TBs": achieved / 8000.0,
+                     "avg_launch_ms_by_step_since_sort": by_step},
         "clocks": clocks,
         "gpu_launches": launches,
         "e2e": e2e,

@@ -24,10 +24,10 @@ namespace {
 
 constexpr int NT = 256;             // threads per radix CTA
 constexpr int NW = NT / 32;         // warps
-constexpr int IPT = 32;             // items per thread
-constexpr int TILE = NT * IPT;      // 8192 elements per tile
-constexpr int MAX_BITS = 13;        // digit width limit (smem: NW * 2^13 * 2 B = 128 KB)
-constexpr int MAX_PASSES = 3;
+constexpr int IPT = 16;             // items per thread
+constexpr int TILE = NT * IPT;      // 4096 elements per tile
+constexpr int MAX_BITS = 8;         // digit width: 256 buckets, one look-back chain per thread
+constexpr int MAX_PASSES = 4;       // keys up to 32 bits
 constexpr unsigned FULL = 0xffffffffu;
 
 constexpr unsigned long long FLAG_AGG = 1ull << 62;
@@ -54,20 +54,12 @@ struct PassDesc {
   int npass;
 };
 
-// ---------------------------------------------------------------- a1 --
-// keys[i] = p_in[i].i ; digit histograms of every pass (warp-aggregated smem
-// counters, one global atomic per non-empty bin per CTA); optional raw
-// new_keys (STANDARD / NONE).
+// keys[i] = p_in[i].i and the voxel histogram count[k] (zeroed by the caller).
+// Runs of equal keys within a warp (the input is nearly sorted between sorts)
+// are counted with one atomic per run, found with a lane-neighbour compare.
 __global__ void __launch_bounds__(256)
-k_keys_hist(const vpic_particle_t *__restrict__ p, int64_t n, uint32_t *__restrict__ keys,
-            PassDesc pd, uint32_t *__restrict__ ghist /*[MAX_PASSES][1<<MAX_BITS]*/,
-            int64_t *__restrict__ new_keys) {
-  extern __shared__ uint32_t sh[];  // [npass][1<<bits_q] (packed)
-  int off[MAX_PASSES];
-  int tot = 0;
-  for (int q = 0; q < pd.npass; ++q) { off[q] = tot; tot += 1 << pd.bits[q]; }
-  for (int i = threadIdx.x; i < tot; i += blockDim.x) sh[i] = 0;
-  __syncthreads();
+k_keys_count(const vpic_particle_t *__restrict__ p, int64_t n, uint32_t *__restrict__ keys,
+             uint32_t *__restrict__ count, int64_t *__restrict__ new_keys) {
   const int lane = threadIdx.x & 31;
   const int32_t *pi = reinterpret_cast<const int32_t *>(p) + 3;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
@@ -75,24 +67,113 @@ k_keys_hist(const vpic_particle_t *__restrict__ p, int64_t n, uint32_t *__restri
        base += stride) {
     const int64_t i = base + lane;
     const bool valid = i < n;
-    uint32_t k = 0;
+    uint32_t k = 0xffffffffu;
     if (valid) {
       k = (uint32_t)__ldcs(pi + 8 * i);
       keys[i] = k;
       if (new_keys) new_keys[i] = (int64_t)k;
     }
-    for (int q = 0; q < pd.npass; ++q) {
-      const uint32_t d = valid ? ((k >> pd.shift[q]) & ((1u << pd.bits[q]) - 1)) : 0xffffffffu;
-      const unsigned peers = __match_any_sync(FULL, d);
-      if (valid && (__ffs(peers) - 1) == lane) atomicAdd(&sh[off[q] + d], __popc(peers));
-    }
+    const uint32_t prev = __shfl_up_sync(FULL, k, 1);
+    const bool head = valid && (lane == 0 || prev != k);
+    const unsigned ends = __ballot_sync(FULL, head) | ~__ballot_sync(FULL, valid);
+    const unsigned above = lane == 31 ? 0u : (ends & ~((2u << lane) - 1u));
+    const int len = (above ? __ffs(above) - 1 : 32) - lane;
+    if (head) atomicAdd(&count[k], (uint32_t)len);
+  }
+}
+
+// Digit histograms of every LSD pass from the voxel histogram.
+__global__ void k_digit_hist(const uint32_t *__restrict__ count, int64_t nv, PassDesc pd,
+                             uint32_t *__restrict__ ghist) {
+  __shared__ uint32_t sh[MAX_PASSES << MAX_BITS];
+  for (int i = threadIdx.x; i < (MAX_PASSES << MAX_BITS); i += blockDim.x) sh[i] = 0;
+  __syncthreads();
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < nv;
+       k += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t c = count[k];
+    if (!c) continue;
+    for (int q = 0; q < pd.npass; ++q)
+      atomicAdd(&sh[(q << MAX_BITS) + (((uint32_t)k >> pd.shift[q]) & ((1u << pd.bits[q]) - 1))], c);
   }
   __syncthreads();
   for (int q = 0; q < pd.npass; ++q)
     for (int b = threadIdx.x; b < (1 << pd.bits[q]); b += blockDim.x) {
-      const uint32_t c = sh[off[q] + b];
-      if (c) atomicAdd(&ghist[q * (1 << MAX_BITS) + b], c);
+      const uint32_t c = sh[(q << MAX_BITS) + b];
+      if (c) atomicAdd(&ghist[(q << MAX_BITS) + b], c);
     }
+}
+
+// offs[k] = sum of count[k' < k] over nv voxels (+ offs[nv] = total), in
+// three phases over blocks of SCAN_B voxels; max_r = max count.
+constexpr int SCAN_B = 4096;
+__global__ void k_scan_blocksum(const uint32_t *__restrict__ count, int64_t nv,
+                                uint32_t *__restrict__ bsum, unsigned int *__restrict__ max_r) {
+  __shared__ uint32_t red[32];
+  __shared__ uint32_t redm[32];
+  const int64_t b0 = (int64_t)blockIdx.x * SCAN_B;
+  uint32_t sum = 0, mx = 0;
+  for (int j = threadIdx.x; j < SCAN_B; j += blockDim.x) {
+    const int64_t k = b0 + j;
+    const uint32_t c = k < nv ? count[k] : 0u;
+    sum += c;
+    mx = max(mx, c);
+  }
+  for (int o = 16; o; o >>= 1) {
+    sum += __shfl_xor_sync(FULL, sum, o);
+    mx = max(mx, __shfl_xor_sync(FULL, mx, o));
+  }
+  if ((threadIdx.x & 31) == 0) { red[threadIdx.x >> 5] = sum; redm[threadIdx.x >> 5] = mx; }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t t = 0, m = 0;
+    for (int w = 0; w < (int)(blockDim.x >> 5); ++w) { t += red[w]; m = max(m, redm[w]); }
+    bsum[blockIdx.x] = t;
+    if (m) atomicMax(max_r, m);
+  }
+}
+__global__ void k_scan_bsums(uint32_t *__restrict__ bsum, int64_t nb) {
+  // one CTA of 1024 threads: exclusive scan in place
+  __shared__ uint32_t part[1024];
+  const int64_t per = (nb + blockDim.x - 1) / blockDim.x;
+  const int64_t j0 = threadIdx.x * per;
+  uint32_t t = 0;
+  for (int64_t j = j0; j < min(nb, j0 + per); ++j) t += bsum[j];
+  part[threadIdx.x] = t;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t run = 0;
+    for (int w = 0; w < (int)blockDim.x; ++w) { const uint32_t x = part[w]; part[w] = run; run += x; }
+  }
+  __syncthreads();
+  uint32_t run = part[threadIdx.x];
+  for (int64_t j = j0; j < min(nb, j0 + per); ++j) { const uint32_t x = bsum[j]; bsum[j] = run; run += x; }
+}
+__global__ void __launch_bounds__(256)
+k_scan_apply(const uint32_t *__restrict__ count, int64_t nv, const uint32_t *__restrict__ bsum,
+             uint32_t *__restrict__ offs, int64_t total) {
+  // 256 threads x 16 consecutive voxels each
+  __shared__ uint32_t wsum[8];
+  const int64_t b0 = (int64_t)blockIdx.x * SCAN_B + threadIdx.x * 16;
+  uint32_t c[16], t = 0;
+#pragma unroll
+  for (int j = 0; j < 16; ++j) { c[j] = (b0 + j < nv) ? count[b0 + j] : 0u; t += c[j]; }
+  uint32_t incl = t;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(FULL, incl, o);
+    if (lane >= o) incl += y;
+  }
+  if (lane == 31) wsum[w] = incl;
+  __syncthreads();
+  uint32_t wpre = 0;
+  for (int ww = 0; ww < w; ++ww) wpre += wsum[ww];
+  uint32_t run = bsum[blockIdx.x] + wpre + incl - t;
+#pragma unroll
+  for (int j = 0; j < 16; ++j) {
+    if (b0 + j < nv) offs[b0 + j] = run;
+    run += c[j];
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) offs[nv] = (uint32_t)total;
 }
 
 // Exclusive scan of each pass's digit histogram (one CTA per pass).
@@ -126,7 +207,7 @@ __global__ void k_scan_hist(const uint32_t *__restrict__ ghist, uint32_t *__rest
 // publishes its per-digit count and resolves its global offset by decoupled
 // look-back over earlier tiles' status words (flag | count in one u64).
 template <int BITS>
-__global__ void __launch_bounds__(NT)
+__global__ void __launch_bounds__(NT, 3)
 k_radix_pass(const uint32_t *__restrict__ kin, const uint32_t *__restrict__ vin,
              uint32_t *__restrict__ kout, uint32_t *__restrict__ vout, int64_t n, int shift,
              const uint32_t *__restrict__ dig_off, unsigned long long *__restrict__ status,
@@ -211,34 +292,6 @@ k_radix_pass(const uint32_t *__restrict__ kin, const uint32_t *__restrict__ vin,
   }
 }
 
-// ---------------------------------------------------------------- counts --
-// offs[k] = first standard-order position with key >= k, k in [0, nv]
-// (lower bound), from the sorted keys; every entry written exactly once.
-__global__ void k_offsets(const uint32_t *__restrict__ K, int64_t n, int64_t nv,
-                          uint32_t *__restrict__ offs) {
-  for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n;
-       j += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t prev = j == 0 ? -1 : (int64_t)K[j - 1];
-    const int64_t cur = K[j];
-    for (int64_t k = prev + 1; k <= cur; ++k) offs[k] = (uint32_t)j;
-    if (j == n - 1)
-      for (int64_t k = cur + 1; k <= nv; ++k) offs[k] = (uint32_t)n;
-  }
-}
-
-__global__ void k_counts(const uint32_t *__restrict__ offs, int64_t nv, int32_t *__restrict__ counts,
-                         unsigned int *__restrict__ max_r) {
-  unsigned int m = 0;
-  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < nv;
-       k += (int64_t)gridDim.x * blockDim.x) {
-    const uint32_t c = offs[k + 1] - offs[k];
-    if (counts) counts[k] = (int32_t)c;
-    m = max(m, c);
-  }
-  for (int o = 16; o; o >>= 1) m = max(m, __shfl_xor_sync(FULL, m, o));
-  if ((threadIdx.x & 31) == 0 && m) atomicMax(max_r, m);
-}
-
 // Rank-pass keys (strided: r; tiled: (chunk - chunk0) * max_r + r) with the
 // digit histograms of the following passes; optional Alg. 1/2 new keys
 // scattered to the INPUT index (perm_std[j]).
@@ -292,15 +345,16 @@ k_rank_keys(const uint32_t *__restrict__ K, const uint32_t *__restrict__ perm_st
 __global__ void __launch_bounds__(256)
 k_gather(const vpic_particle_t *__restrict__ pin, vpic_particle_t *__restrict__ pout,
          const uint32_t *__restrict__ perm, int64_t n, int64_t *__restrict__ perm64) {
+  // two threads per 32-B record: every warp load / store instruction moves
+  // 16 whole records (sector-complete) and the stores are fully coalesced
   const float4 *src = reinterpret_cast<const float4 *>(pin);
   float4 *dst = reinterpret_cast<float4 *>(pout);
-  for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < n;
+  for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < 2 * n;
        t += (int64_t)gridDim.x * blockDim.x) {
-    const uint32_t s = perm[t];
-    const float4 a = __ldcs(src + 2 * (int64_t)s), b = __ldcs(src + 2 * (int64_t)s + 1);
-    __stcs(dst + 2 * t, a);
-    __stcs(dst + 2 * t + 1, b);
-    if (perm64) perm64[t] = s;
+    const int64_t r = t >> 1;
+    const uint32_t sidx = __ldg(perm + r);
+    __stcs(dst + t, __ldcs(src + 2 * (int64_t)sidx + (t & 1)));
+    if (perm64 && !(t & 1)) perm64[r] = sidx;
   }
 }
 
@@ -327,7 +381,7 @@ __global__ void k_hist_voxels(const vpic_particle_t *__restrict__ p, int64_t n,
 
 // ------------------------------------------------------------ host side --
 struct WsLayout {
-  size_t keysA, keysB, valsA, valsB, offs, ghist, goff, status, ctr, misc, total;
+  size_t keysA, keysB, valsA, valsB, offs, count, bsum, ghist, goff, status, ctr, misc, total;
 };
 
 inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
@@ -342,6 +396,8 @@ WsLayout layout(int64_t np, int64_t nv) {
   L.valsA = take(4 * (size_t)np);
   L.valsB = take(4 * (size_t)np);
   L.offs = take(4 * (size_t)(nv + 1));
+  L.count = take(4 * (size_t)nv);
+  L.bsum = take(4 * (size_t)(nv / SCAN_B + 2));
   L.ghist = take(4 * (size_t)MAX_PASSES * (1 << MAX_BITS));
   L.goff = take(4 * (size_t)MAX_PASSES * (1 << MAX_BITS));
   L.status = take(8 * (size_t)std::max<int64_t>(tiles, 1) * (1 << MAX_BITS));
@@ -393,8 +449,7 @@ cudaError_t radix_pass(int bits, const uint32_t *kin, const uint32_t *vin, uint3
                        unsigned long long *status, unsigned int *ctr, cudaStream_t s) {
   switch (bits) {
 #define VPIC_RP(B) case B: return radix_pass_bits<B>(kin, vin, kout, vout, n, shift, dig_off, status, ctr, s);
-    VPIC_RP(1) VPIC_RP(2) VPIC_RP(3) VPIC_RP(4) VPIC_RP(5) VPIC_RP(6) VPIC_RP(7)
-    VPIC_RP(8) VPIC_RP(9) VPIC_RP(10) VPIC_RP(11) VPIC_RP(12) VPIC_RP(13)
+    VPIC_RP(1) VPIC_RP(2) VPIC_RP(3) VPIC_RP(4) VPIC_RP(5) VPIC_RP(6) VPIC_RP(7) VPIC_RP(8)
 #undef VPIC_RP
     default: return cudaErrorInvalidValue;
   }
@@ -480,31 +535,28 @@ cudaError_t launch_sort(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_
   unsigned int *ctr = reinterpret_cast<unsigned int *>(w + L.ctr);
   unsigned int *misc = reinterpret_cast<unsigned int *>(w + L.misc);
 
-  // ---- standard order: stable LSD radix sort by voxel
+  // ---- voxel histogram (deterministic run counts), digit histograms
+  uint32_t *count = voxel_counts ? reinterpret_cast<uint32_t *>(voxel_counts)
+                                 : reinterpret_cast<uint32_t *>(w + L.count);
+  CK(cudaMemsetAsync(count, 0, 4 * (size_t)nv, s));
+  k_keys_count<<<grid_cap(np, 256, sms, 8), 256, 0, s>>>(
+      p_in, np, kA, count, (order == VPIC_SORT_STANDARD) ? new_keys : nullptr); note_launch();
+  CK(cudaGetLastError());
   const PassDesc pd = make_passes(bits_for((uint64_t)(nv - 1)));
   CK(cudaMemsetAsync(ghist, 0, 4 * (size_t)MAX_PASSES * (1 << MAX_BITS), s));
-  {
-    int tot = 0;
-    for (int q = 0; q < pd.npass; ++q) tot += 1 << pd.bits[q];
-    const size_t smem = 4 * (size_t)tot;
-    static bool configured = false;
-    if (!configured) {
-      cudaFuncSetAttribute(k_keys_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, 4 * 3 * 8192);
-      configured = true;
-    }
-    k_keys_hist<<<grid_cap(np, 256, sms, 2), 256, smem, s>>>(
-        p_in, np, kA, pd, ghist, (order == VPIC_SORT_STANDARD) ? new_keys : nullptr); note_launch();
-    CK(cudaGetLastError());
-  }
+  k_digit_hist<<<grid_cap(nv, 256, sms, 2), 256, 0, s>>>(count, nv, pd, ghist); note_launch();
+  CK(cudaGetLastError());
+  // ---- standard order: stable LSD radix sort of (voxel, index)
   uint32_t *K = nullptr, *P = nullptr;
-  const bool need_offs = (order != VPIC_SORT_STANDARD) || voxel_counts;
+  const bool need_offs = order != VPIC_SORT_STANDARD;
   CK(lsd_sort(pd, np, kA, kB, vA, vB, nullptr, ghist, goff, status, ctr, need_offs, &K, &P, s));
-
-  if (need_offs) {
-    k_offsets<<<grid_cap(np, 256, sms, 16), 256, 0, s>>>(K, np, nv, offs); note_launch();
-    CK(cudaGetLastError());
+  if (need_offs) {  // offs[k] = first standard position of voxel k; max_r
+    uint32_t *bsum = reinterpret_cast<uint32_t *>(w + L.bsum);
+    const int64_t nb = (nv + SCAN_B - 1) / SCAN_B;
     CK(cudaMemsetAsync(misc, 0, 64, s));
-    k_counts<<<grid_cap(nv, 256, sms, 16), 256, 0, s>>>(offs, nv, voxel_counts, misc); note_launch();
+    k_scan_blocksum<<<(unsigned)nb, 256, 0, s>>>(count, nv, bsum, misc); note_launch();
+    k_scan_bsums<<<1, 1024, 0, s>>>(bsum, nb); note_launch();
+    k_scan_apply<<<(unsigned)nb, 256, 0, s>>>(count, nv, bsum, offs, np); note_launch();
     CK(cudaGetLastError());
   }
   if (order == VPIC_SORT_STRIDED || order == VPIC_SORT_TILED_STRIDED) {
@@ -531,7 +583,7 @@ cudaError_t launch_sort(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_
       for (int q = 0; q < pr.npass; ++q) tot += 1 << pr.bits[q];
       static bool configured = false;
       if (!configured) {
-        cudaFuncSetAttribute(k_rank_keys, cudaFuncAttributeMaxDynamicSharedMemorySize, 4 * 3 * 8192);
+        cudaFuncSetAttribute(k_rank_keys, cudaFuncAttributeMaxDynamicSharedMemorySize, 4 * MAX_PASSES * (1 << MAX_BITS));
         configured = true;
       }
       k_rank_keys<<<grid_cap(np, 256, sms, 2), 256, 4 * (size_t)tot, s>>>(
@@ -545,7 +597,7 @@ cudaError_t launch_sort(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_
     CK(lsd_sort(pr, np, kX, kY, vX, vY, P, ghist, goff, status, ctr, false, &K2, &P2, s));
     P = P2;
   }
-  k_gather<<<grid_cap(np, 256, sms, 16), 256, 0, s>>>(p_in, p_out, P, np, perm); note_launch();
+  k_gather<<<grid_cap(2 * np, 256, sms, 16), 256, 0, s>>>(p_in, p_out, P, np, perm); note_launch();
   return cudaGetLastError();
 }
 

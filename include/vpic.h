@@ -20,9 +20,11 @@
  *      particle      vpic_particle_t, 32 B (AoS);
  *      fields[nv][8] float: ex,ey,ez,0, cbx,cby,cbz,0 (Yee: ex on the x-edge
  *                    from node (x,y,z) to (x+1,y,z), cbx on the -x face);
- *      interp[nv][20] float: ex,dexdy,dexdz,d2exdydz, ey,deydz,deydx,
+ *      interp[nv][24] float: ex,dexdy,dexdz,d2exdydz, ey,deydz,deydx,
  *                    d2eydzdx, ez,dezdx,dezdy,d2ezdxdy, cbx,dcbxdx,
- *                    cby,dcbydy, cbz,dcbzdz, 0,0  (80 B = 5 x float4);
+ *                    cby,dcbydy, cbz,dcbzdz, then 6 zero pads (96 B = three
+ *                    32-B sectors, so a gather is three 256-bit loads);
+ *                    the array must be 32-B aligned;
  *      acc[nv][12]   float: jx[4], jy[4], jz[4] quadrant partials
  *                    (48 B = 3 x float4); jx quadrants (-y-z),(+y-z),(-y+z),(+y+z),
  *                    jy cyclic over (z,x), jz over (x,y);
@@ -150,7 +152,7 @@ int vpic_sort_particles(vpic_ctx *ctx, const vpic_particle_t *p_in, vpic_particl
  * place, then write interp[v] for every interior voxel v (ghost voxels of
  * interp are left untouched).  Ghost planes of REFLECT/ABSORB faces are the
  * caller's. */
-int vpic_load_interpolator(vpic_ctx *ctx, float *fields, float *interp, void *stream);
+int vpic_load_interpolator(vpic_ctx *ctx, float *fields, float *interp /*[nv][24]*/, void *stream);
 
 /* ------------------------------------------------ (a6) clear accumulator -- */
 int vpic_clear_accumulator(vpic_ctx *ctx, float *acc, void *stream);

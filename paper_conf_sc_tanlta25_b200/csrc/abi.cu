@@ -14,6 +14,7 @@ using namespace vpic;
 namespace {
 
 bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+bool aligned32(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 31u) == 0; }
 
 cudaStream_t S(void *s) { return static_cast<cudaStream_t>(s); }
 
@@ -215,7 +216,7 @@ int vpic_sort_particles(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_
 }
 
 int vpic_load_interpolator(vpic_ctx *c, float *fields, float *interp, void *stream) {
-  if (!c || !fields || !interp || !aligned16(fields) || !aligned16(interp)) return VPIC_ERR_INVALID;
+  if (!c || !fields || !interp || !aligned16(fields) || !aligned32(interp)) return VPIC_ERR_INVALID;
   DeviceGuard dg(c->device);
   cudaError_t e = launch_fill_ghosts(c, fields, S(stream));
   if (e != cudaSuccess) return VPIC_ERR_CUDA;
@@ -237,7 +238,7 @@ int vpic_advance_p(vpic_ctx *c, float q, float m, vpic_particle_t *p, int64_t np
                    int64_t *n_movers, int32_t *flags, void *stream) {
   if (!c || np < 0 || np >= ((int64_t)1 << 31) || !(m > 0) || max_movers < 0) return VPIC_ERR_INVALID;
   if (np == 0) return VPIC_OK;
-  if (!p || !interp || !acc || !n_movers || !aligned16(p) || !aligned16(interp) || !aligned16(acc))
+  if (!p || !interp || !acc || !n_movers || !aligned16(p) || !aligned32(interp) || !aligned16(acc))
     return VPIC_ERR_INVALID;
   if (max_movers > 0 && (!movers || !aligned16(movers))) return VPIC_ERR_INVALID;
   if ((reinterpret_cast<uintptr_t>(n_movers) & 7u) != 0) return VPIC_ERR_INVALID;

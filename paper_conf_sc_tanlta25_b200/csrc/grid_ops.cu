@@ -30,7 +30,8 @@ __global__ void k_fill_ghosts(const GridK g, const Per per, float4 *__restrict__
 }
 
 // One thread per interior voxel; a CTA covers a run of x along one (y,z) row
-// so the x+1 neighbours come from L1.  interp[v] = 5 x float4 (80 B).
+// so the x+1 neighbours come from L1.  interp[v] = 6 x float4 (96 B, the last
+// 24 B zero) so that a particle's gather is three sector-aligned 32-B loads.
 __global__ void __launch_bounds__(128)
 k_load_interp(const GridK g, const float4 *__restrict__ f, float4 *__restrict__ interp) {
   const int nrows = g.ny * g.nz;
@@ -79,8 +80,9 @@ k_load_interp(const GridK g, const float4 *__restrict__ f, float4 *__restrict__ 
     o4.y = half * (b001.z - b000.z);
     o4.z = 0.0f;
     o4.w = 0.0f;
-    float4 *o = interp + 5 * v;
+    float4 *o = interp + 6 * v;
     o[0] = o0; o[1] = o1; o[2] = o2; o[3] = o3; o[4] = o4;
+    o[5] = make_float4(0.f, 0.f, 0.f, 0.f);
   }
 }
 

@@ -52,7 +52,7 @@ class HotPath:
         nv = self.g.nv
         f32 = dict(dtype=torch.float32, device=self.dev)
         self.fields = torch.from_numpy(np.ascontiguousarray(fields)).to(self.dev)
-        self.interp = torch.zeros((nv, 20), **f32)
+        self.interp = torch.zeros((nv, 24), **f32)
         self.acc = torch.zeros((nv, 12), **f32)
         self.jf = torch.zeros((nv, 4), **f32)
         self.species: List[SpeciesState] = []

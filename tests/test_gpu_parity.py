@@ -130,7 +130,7 @@ def run_both(V, orc, g, p, q, m, fields, math, deposit, kernel=0):
     mv_o = orc.advance_p(g, q, m, p_o, interp_o, acc_o, acc_abs)
     ctx = mkctx(V, g, math, deposit, kernel)
     fd = torch.from_numpy(fields.copy()).cuda()
-    interp = torch.zeros((g.nv, 20), dtype=torch.float32, device="cuda")
+    interp = torch.zeros((g.nv, 24), dtype=torch.float32, device="cuda")
     V.vpic_load_interpolator(ctx, fd, interp)
     acc = torch.empty((g.nv, 12), dtype=torch.float32, device="cuda")
     V.vpic_clear_accumulator(ctx, acc)
@@ -153,7 +153,8 @@ def test_advance_ieee_bitexact(V, orc, case, deposit, kernel):
     name, g, p, q, m, f = case
     r = run_both(V, orc, g, p, q, m, f, V.MATH_IEEE, deposit, kernel)
     vox = g.interior_voxels()
-    assert np.array_equal(r["interp"][vox], r["interp_o"][vox])
+    assert np.array_equal(r["interp"][vox, :20], r["interp_o"][vox])
+    assert np.all(r["interp"][vox, 20:] == 0)
     assert_particles_bitexact(r["p"], r["p_o"])
     assert_acc_close(r["acc"], r["acc_o"], r["acc_abs"])
     assert r["nm"] == 0 and r["flags"] == 0
@@ -245,7 +246,7 @@ def test_mover_overflow_flag(V, orc):
     p = inputs.random_particles(g, 9000, 31, u_scale=1.5)
     ctx = mkctx(V, g)
     fd = torch.from_numpy(inputs.make_fields(g, 0.01)).cuda()
-    interp = torch.zeros((g.nv, 20), device="cuda")
+    interp = torch.zeros((g.nv, 24), device="cuda")
     V.vpic_load_interpolator(ctx, fd, interp)
     acc = torch.zeros((g.nv, 12), device="cuda")
     pd = dev_particles(V, p)

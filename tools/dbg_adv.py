@@ -10,7 +10,7 @@ ctx = vpic.Context(g)
 ctx.set_option(vpic.VPIC_OPT_ADVANCE_KERNEL, 2)
 ctx.set_option(vpic.VPIC_OPT_DEPOSIT, 2)
 fd = torch.from_numpy(inputs.make_fields(g, 0.01)).cuda()
-interp = torch.zeros((g.nv, 20), device="cuda")
+interp = torch.zeros((g.nv, 24), device="cuda")
 vpic.vpic_load_interpolator(ctx, fd, interp)
 acc = torch.zeros((g.nv, 12), device="cuda")
 pd = vpic.particles_to_device(p)

@@ -166,6 +166,11 @@ def run_oracle_steps(wl, n_steps, sort_every, order):
     return times, sum(p.size for p in parts) * sort_every
 
 
+def inputs_config_name(args):
+    from paper_conf_sc_tanlta25_b200 import inputs
+    return inputs.config(args.config).name
+
+
 def reference_arm(args, rank, world):
     if rank != 0:
         return
@@ -181,8 +186,8 @@ def reference_arm(args, rank, world):
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * total / args.steps,
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
         "data": "synthetic",
-        "config": {"workload": wl.name, "order": args.order, "sort_every": S,
-                   "particles": per_step // S},
+        "config": {"workload": inputs_config_name(args), "order": args.order, "sort_every": S,
+                   "sample": f"{wl.name}: {per_step // S} particles per step (bounded CPU sample)"},
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
                          "sample": f"serial C++ oracle (oracle/), {wl.name}: {per_step // S} particles, "
                                    f"sort + {S} PIC steps per step"},

@@ -343,7 +343,7 @@ def our_arm(args, rank, world):
                    "species": len(wl.species), "particles": int(ntot), "sort_every": S,
                    "order": args.order, "shuffled": bool(args.shuffle), "math": args.math,
                    "deposit": args.deposit, "kernel": args.kernel, "parallelism": f"domain{world}",
-                   "l2": "no flush: inputs (17 GB of particles per GPU) >> 126 MB L2"},
+                   "l2": f"no flush: inputs ({32 * n_local / 1e9:.1f} GB of particles per GPU) >> 126 MB L2"},
         "per_gpu": value / world,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,

@@ -300,18 +300,7 @@ def our_arm(args, rank, world):
         barrier()
         a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a0.record(stream)
-        e2e_pushes = 0
-        for _ in range(args.steps):
-            for s, h in zip(hp.species, host_in):
-                s.p[:h.shape[0]].copy_(h, non_blocking=True)
-                s.np = h.shape[0]
-            hp.fields.copy_(f_host, non_blocking=True)
-            hp.cycle(S)
-            e2e_pushes += S * hp.n_particles
-            for s, h in zip(hp.species, host_out):
-                n = min(s.np, h.shape[0])
-                h[:n].copy_(s.p[:n], non_blocking=True)
-            jf_host.copy_(hp.jf, non_blocking=True)
+        e2e_pushes = hp.run_host_cycles(host_in, host_out, f_host, jf_host, args.steps, S)
         a1.record(stream)
         torch.cuda.synchronize()
         barrier()

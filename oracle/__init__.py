@@ -76,6 +76,10 @@ def lib() -> ctypes.CDLL:
         _lib.orc_accumulate_rho.restype = None
         _lib.orc_remove_absorbed.argtypes = [G, P, I64, P, I64]
         _lib.orc_remove_absorbed.restype = I64
+        _lib.orc_advance_b.argtypes = [G, P, ctypes.c_float]
+        _lib.orc_advance_b.restype = None
+        _lib.orc_advance_e.argtypes = [G, P, P, ctypes.c_float]
+        _lib.orc_advance_e.restype = None
     return _lib
 
 
@@ -184,3 +188,18 @@ def remove_absorbed(spec, p, movers):
     g = make_grid(spec)
     n = lib().orc_remove_absorbed(ctypes.byref(g), _ptr(p), p.size, _ptr(movers), movers.size)
     return p[:n].copy()
+
+
+# ------------------------------------------------------------ field solver --
+def advance_b(spec, fields, frac):
+    """In place on fields float32[nv, 8] (ghost planes refreshed)."""
+    assert fields.dtype == np.float32 and fields.flags.c_contiguous
+    g = make_grid(spec)
+    lib().orc_advance_b(ctypes.byref(g), _ptr(fields), frac)
+
+
+def advance_e(spec, fields, jf, eps0=1.0):
+    assert fields.dtype == np.float32 and fields.flags.c_contiguous
+    jf = np.ascontiguousarray(jf, dtype=np.float32)
+    g = make_grid(spec)
+    lib().orc_advance_e(ctypes.byref(g), _ptr(fields), _ptr(jf), eps0)

@@ -88,6 +88,15 @@ void orc_accumulate_rho(const orc_grid *g, const orc_particle *p, int64_t np, fl
 int64_t orc_remove_absorbed(const orc_grid *g, orc_particle *p, int64_t np,
                             const orc_mover *movers, int64_t n_movers);
 
+/* Field solver (VPIC ref. [3] advance_b / advance_e,
+ * reading F1 in DESIGN.md).  fields[nv][8] = ex,ey,ez,0,cbx,cby,cbz,0.
+ * Ghost planes of locally periodic axes are refreshed first (E at +1 planes
+ * for advance_b, cB at -1 planes for advance_e); interior voxels updated.
+ *   advance_b: cB -= frac c dt curl E      (forward differences)
+ *   advance_e: E  += c dt curl cB - (dt/eps0) jf   (backward differences) */
+void orc_advance_b(const orc_grid *g, float *fields, float frac);
+void orc_advance_e(const orc_grid *g, float *fields, const float *jf, float eps0);
+
 #ifdef __cplusplus
 }
 #endif

@@ -183,6 +183,21 @@ int vpic_advance_p(vpic_ctx *ctx, float q, float m, vpic_particle_t *p, int64_t 
  * n+1 ghost copies made equal to plane 1.  jf is overwritten. */
 int vpic_unload_accumulator(vpic_ctx *ctx, const float *acc, float *jf, void *stream);
 
+/* ------------------------------------------- (f1) field solver (next row) -- */
+
+/* Yee field advance of VPIC (ref. [3]; SURVEY.md §8(f) f1 -- "full simulation"
+ * runtime is a paper metric).  fields[nv][8] as above, updated in
+ * place on interior voxels; locally periodic ghost planes are refreshed (and
+ * remote ones exchanged over NCCL) first.
+ *   vpic_advance_b: cB -= frac * c dt curl E (forward differences; needs the
+ *                   +x/+y/+z ghost planes of E);
+ *   vpic_advance_e: E += c dt curl cB - (dt/eps0) jf (backward differences;
+ *                   needs the -x/-y/-z ghost planes of cB), jf[nv][4] from
+ *                   vpic_unload_accumulator.
+ * A VPIC step is advance_b(1/2), advance_e, advance_b(1/2). */
+int vpic_advance_b(vpic_ctx *ctx, float *fields, float frac, void *stream);
+int vpic_advance_e(vpic_ctx *ctx, float *fields, const float *jf, float eps0, void *stream);
+
 /* ---------------------------------------------------- (a13) exchange -- */
 
 /* Finish the movers produced by vpic_advance_p for one species: particles on

@@ -221,7 +221,7 @@ int vpic_load_interpolator(vpic_ctx *c, float *fields, float *interp, void *stre
   cudaError_t e = launch_fill_ghosts(c, fields, S(stream));
   if (e != cudaSuccess) return VPIC_ERR_CUDA;
   if (c->ex) {
-    const int rc = halo_fields(c, fields, S(stream));
+    const int rc = halo_fields(c, fields, S(stream), +1);
     if (rc != VPIC_OK) return rc;
   }
   return cuda_status(launch_load_interp(c, fields, interp, S(stream)));
@@ -255,6 +255,29 @@ int vpic_unload_accumulator(vpic_ctx *c, const float *acc, float *jf, void *stre
   if (e != cudaSuccess) return VPIC_ERR_CUDA;
   if (c->ex) return reduce_jf(c, jf, S(stream));
   return VPIC_OK;
+}
+
+int vpic_advance_b(vpic_ctx *c, float *fields, float frac, void *stream) {
+  if (!c || !fields || !aligned16(fields) || !(frac >= 0)) return VPIC_ERR_INVALID;
+  DeviceGuard dg(c->device);
+  if (launch_fill_ghosts(c, fields, S(stream)) != cudaSuccess) return VPIC_ERR_CUDA;
+  if (c->ex) {
+    const int rc = halo_fields(c, fields, S(stream), +1);
+    if (rc != VPIC_OK) return rc;
+  }
+  return cuda_status(launch_advance_b(c, fields, frac, S(stream)));
+}
+
+int vpic_advance_e(vpic_ctx *c, float *fields, const float *jf, float eps0, void *stream) {
+  if (!c || !fields || !jf || !aligned16(fields) || !aligned16(jf) || !(eps0 > 0))
+    return VPIC_ERR_INVALID;
+  DeviceGuard dg(c->device);
+  if (launch_fill_ghosts_minus(c, fields, S(stream)) != cudaSuccess) return VPIC_ERR_CUDA;
+  if (c->ex) {
+    const int rc = halo_fields(c, fields, S(stream), -1);
+    if (rc != VPIC_OK) return rc;
+  }
+  return cuda_status(launch_advance_e(c, fields, jf, eps0, S(stream)));
 }
 
 int vpic_migrate_particles(vpic_ctx *c, float q, float m, vpic_particle_t *p, int64_t *np,

@@ -29,6 +29,69 @@ __global__ void k_fill_ghosts(const GridK g, const Per per, float4 *__restrict__
   }
 }
 
+// -x/-y/-z ghost planes of locally periodic axes := copy of plane n (the cB
+// neighbours advance_e needs).  Same direct mapping as k_fill_ghosts.
+__global__ void k_fill_ghosts_minus(const GridK g, const Per per, float4 *__restrict__ f) {
+  const int64_t nv = g.nv;
+  for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < nv;
+       v += (int64_t)gridDim.x * blockDim.x) {
+    int x = (int)(v % g.sx), y = (int)((v / g.sx) % g.sy), z = (int)(v / g.sxy);
+    bool w = false;
+    if (per.px && x == 0) { x = g.nx; w = true; }
+    if (per.py && y == 0) { y = g.ny; w = true; }
+    if (per.pz && z == 0) { z = g.nz; w = true; }
+    if (!w) continue;
+    const int64_t src = x + (int64_t)g.sx * (y + (int64_t)g.sy * z);
+    f[2 * v] = f[2 * src];
+    f[2 * v + 1] = f[2 * src + 1];
+  }
+}
+
+// Field solver (VPIC advance_b / advance_e, reading F1):
+// one thread per interior voxel, consecutive threads along x.
+//   advance_b: cB -= frac c dt curl E   (E at +1 neighbours)
+//   advance_e: E  += c dt curl cB - (dt/eps0) jf   (cB at -1 neighbours)
+// Same expressions and order as the oracle; compiled without FMA contraction.
+__global__ void __launch_bounds__(256)
+k_advance_b(const GridK g, const float px, const float py, const float pz, float4 *__restrict__ f) {
+  const int64_t ncell = (int64_t)g.nx * g.ny * g.nz;
+  for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < ncell;
+       t += (int64_t)gridDim.x * blockDim.x) {
+    const int x = 1 + (int)(t % g.nx);
+    const int row = (int)(t / g.nx);
+    const int y = 1 + row % g.ny, z = 1 + row / g.ny;
+    const int64_t v = x + (int64_t)g.sx * (y + (int64_t)g.sy * z);
+    const float4 e = f[2 * v];
+    float4 b = f[2 * v + 1];
+    const float4 ex1 = f[2 * (v + 1)], ey1 = f[2 * (v + g.sx)], ez1 = f[2 * (v + g.sxy)];
+    b.x -= py * (ey1.z - e.z) - pz * (ez1.y - e.y);
+    b.y -= pz * (ez1.x - e.x) - px * (ex1.z - e.z);
+    b.z -= px * (ex1.y - e.y) - py * (ey1.x - e.x);
+    f[2 * v + 1] = b;
+  }
+}
+
+__global__ void __launch_bounds__(256)
+k_advance_e(const GridK g, const float px, const float py, const float pz, const float cj,
+            float4 *__restrict__ f, const float4 *__restrict__ jf) {
+  const int64_t ncell = (int64_t)g.nx * g.ny * g.nz;
+  for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < ncell;
+       t += (int64_t)gridDim.x * blockDim.x) {
+    const int x = 1 + (int)(t % g.nx);
+    const int row = (int)(t / g.nx);
+    const int y = 1 + row % g.ny, z = 1 + row / g.ny;
+    const int64_t v = x + (int64_t)g.sx * (y + (int64_t)g.sy * z);
+    float4 e = f[2 * v];
+    const float4 b = f[2 * v + 1];
+    const float4 bx1 = f[2 * (v - 1) + 1], by1 = f[2 * (v - g.sx) + 1], bz1 = f[2 * (v - g.sxy) + 1];
+    const float4 j = __ldg(jf + v);
+    e.x += py * (b.z - by1.z) - pz * (b.y - bz1.y) - cj * j.x;
+    e.y += pz * (b.x - bz1.x) - px * (b.z - bx1.z) - cj * j.y;
+    e.z += px * (b.y - bx1.y) - py * (b.x - by1.x) - cj * j.z;
+    f[2 * v] = e;
+  }
+}
+
 // One thread per interior voxel; a CTA covers a run of x along one (y,z) row
 // so the x+1 neighbours come from L1.  interp[v] = 6 x float4 (96 B, the last
 // 24 B zero) so that a particle's gather is three sector-aligned 32-B loads.
@@ -143,6 +206,40 @@ cudaError_t launch_load_interp(const vpic_ctx *c, const float *fields, float *in
   const int64_t n = (int64_t)c->gk.nx * c->gk.ny * c->gk.nz;
   k_load_interp<<<grid_for(n, 128, c->num_sms), 128, 0, s>>>(
       c->gk, reinterpret_cast<const float4 *>(fields), reinterpret_cast<float4 *>(interp)); note_launch();
+  return cudaGetLastError();
+}
+
+cudaError_t launch_fill_ghosts_minus(const vpic_ctx *c, float *fields, cudaStream_t s) {
+  Per per{c->periodic_local[0], c->periodic_local[1], c->periodic_local[2]};
+  if (!per.px && !per.py && !per.pz) return cudaSuccess;
+  k_fill_ghosts_minus<<<grid_for(c->gk.nv, 256, c->num_sms), 256, 0, s>>>(
+      c->gk, per, reinterpret_cast<float4 *>(fields)); note_launch();
+  return cudaGetLastError();
+}
+
+cudaError_t launch_advance_b(const vpic_ctx *c, float *fields, float frac, cudaStream_t s) {
+  const vpic_grid_t &g = c->g;
+  // same expressions as the oracle: frac * c * dt / d
+  const float px = frac * g.cvac * g.dt / g.dx;
+  const float py = frac * g.cvac * g.dt / g.dy;
+  const float pz = frac * g.cvac * g.dt / g.dz;
+  const int64_t n = (int64_t)g.nx * g.ny * g.nz;
+  k_advance_b<<<grid_for(n, 256, c->num_sms), 256, 0, s>>>(c->gk, px, py, pz,
+                                                           reinterpret_cast<float4 *>(fields)); note_launch();
+  return cudaGetLastError();
+}
+
+cudaError_t launch_advance_e(const vpic_ctx *c, float *fields, const float *jf, float eps0,
+                             cudaStream_t s) {
+  const vpic_grid_t &g = c->g;
+  const float px = g.cvac * g.dt / g.dx;
+  const float py = g.cvac * g.dt / g.dy;
+  const float pz = g.cvac * g.dt / g.dz;
+  const float cj = g.dt / eps0;
+  const int64_t n = (int64_t)g.nx * g.ny * g.nz;
+  k_advance_e<<<grid_for(n, 256, c->num_sms), 256, 0, s>>>(c->gk, px, py, pz, cj,
+                                                           reinterpret_cast<float4 *>(fields),
+                                                           reinterpret_cast<const float4 *>(jf)); note_launch();
   return cudaGetLastError();
 }
 

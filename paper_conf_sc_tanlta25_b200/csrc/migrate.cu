@@ -324,9 +324,11 @@ int migrate(vpic_ctx *c, float qsp, float msp, vpic_particle_t *p, int64_t *np_i
   return VPIC_OK;
 }
 
-// E/cB ghost planes from the neighbours: axis by axis, my plane 1 goes to the
-// -face neighbour, whose plane n+1 it fills (edges/corners propagate).
-int halo_fields(vpic_ctx *c, float *fields, cudaStream_t s) {
+// E/cB ghost planes from the neighbours, axis by axis (edges / corners
+// propagate because each plane spans the other axes' ghosts).  dir = +1: my
+// plane 1 goes to the -face neighbour, whose plane n+1 it fills; dir = -1: my
+// plane n goes to the +face neighbour, whose plane 0 it fills.
+int halo_fields(vpic_ctx *c, float *fields, cudaStream_t s, int dir) {
   Exchange *ex = c->ex;
   const GridK &g = c->gk;
   const int sz = g.nz + 2;
@@ -334,17 +336,19 @@ int halo_fields(vpic_ctx *c, float *fields, cudaStream_t s) {
   if (int rc = ensure_plane(ex, maxplane)) return rc;
   for (int axis = 0; axis < 3; ++axis) {
     if (c->periodic_local[axis]) continue;
-    const int fm = axis, fp = axis + 3;
-    const bool send_m = g.face_kind[fm] == FACE_REMOTE, recv_p = g.face_kind[fp] == FACE_REMOTE;
-    if (!send_m && !recv_p) continue;
+    const int f_to = dir > 0 ? axis : axis + 3;     // face whose neighbour receives my plane
+    const int f_from = dir > 0 ? axis + 3 : axis;   // face whose neighbour fills my ghost
+    const bool snd = g.face_kind[f_to] == FACE_REMOTE, rcv = g.face_kind[f_from] == FACE_REMOTE;
+    if (!snd && !rcv) continue;
     const int n = axis == 0 ? g.nx : (axis == 1 ? g.ny : g.nz);
+    const int src_plane = dir > 0 ? 1 : n, dst_plane = dir > 0 ? n + 1 : 0;
     const int64_t cnt = (axis == 0 ? (int64_t)g.sy * sz : axis == 1 ? (int64_t)g.sx * sz : (int64_t)g.sx * g.sy) * 8;
-    if (send_m) { k_plane_copy<<<blocks_for(cnt), 256, 0, s>>>(g, axis, 1, fields, 8, ex->plane_send, 0); note_launch(); }
+    if (snd) { k_plane_copy<<<blocks_for(cnt), 256, 0, s>>>(g, axis, src_plane, fields, 8, ex->plane_send, 0); note_launch(); }
     CKN(ncclGroupStart());
-    if (send_m) CKN(ncclSend(ex->plane_send, cnt, ncclFloat32, c->g.nbr_rank[fm], ex->comm, s));
-    if (recv_p) CKN(ncclRecv(ex->plane_recv, cnt, ncclFloat32, c->g.nbr_rank[fp], ex->comm, s));
+    if (snd) CKN(ncclSend(ex->plane_send, cnt, ncclFloat32, c->g.nbr_rank[f_to], ex->comm, s));
+    if (rcv) CKN(ncclRecv(ex->plane_recv, cnt, ncclFloat32, c->g.nbr_rank[f_from], ex->comm, s));
     CKN(ncclGroupEnd());
-    if (recv_p) { k_plane_copy<<<blocks_for(cnt), 256, 0, s>>>(g, axis, n + 1, fields, 8, ex->plane_recv, 1); note_launch(); }
+    if (rcv) { k_plane_copy<<<blocks_for(cnt), 256, 0, s>>>(g, axis, dst_plane, fields, 8, ex->plane_recv, 1); note_launch(); }
     CKC(cudaGetLastError());
   }
   return VPIC_OK;

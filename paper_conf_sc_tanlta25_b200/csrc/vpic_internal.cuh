@@ -80,6 +80,10 @@ cudaError_t launch_fill_ghosts(const vpic_ctx *c, float *fields, cudaStream_t s)
 cudaError_t launch_load_interp(const vpic_ctx *c, const float *fields, float *interp,
                                cudaStream_t s);
 cudaError_t launch_unload(const vpic_ctx *c, const float *acc, float *jf, cudaStream_t s);
+cudaError_t launch_fill_ghosts_minus(const vpic_ctx *c, float *fields, cudaStream_t s);
+cudaError_t launch_advance_b(const vpic_ctx *c, float *fields, float frac, cudaStream_t s);
+cudaError_t launch_advance_e(const vpic_ctx *c, float *fields, const float *jf, float eps0,
+                             cudaStream_t s);
 
 size_t sort_workspace_bytes(const vpic_ctx *c, int64_t np, int order);
 cudaError_t launch_sort(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_t *p_out,
@@ -91,7 +95,9 @@ int migrate(vpic_ctx *c, float qsp, float msp, vpic_particle_t *p, int64_t *np, 
             vpic_mover_t *movers, const int64_t *n_movers, float *acc, cudaStream_t s);
 int exchange_create(vpic_ctx *c, const uint8_t *uid);
 void exchange_destroy(vpic_ctx *c);
-int halo_fields(vpic_ctx *c, float *fields, cudaStream_t s);
+// dir = +1: fill the +x/+y/+z ghost planes from the +neighbours' plane 1;
+// dir = -1: fill the -x/-y/-z ghost planes from the -neighbours' plane n.
+int halo_fields(vpic_ctx *c, float *fields, cudaStream_t s, int dir = +1);
 int reduce_jf(vpic_ctx *c, float *jf, cudaStream_t s);
 
 }  // namespace vpic

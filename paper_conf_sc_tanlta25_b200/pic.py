@@ -5,6 +5,7 @@ PIC step made only of libvpic C-ABI calls:
     vpic_load_interpolator -> vpic_clear_accumulator
     -> vpic_advance_p (per species) -> [vpic_migrate_particles]
     -> vpic_unload_accumulator
+    [-> vpic_advance_b(1/2) -> vpic_advance_e -> vpic_advance_b(1/2)]   (field_solve)
 
 PyTorch only provides device memory, pinned host memory and the stream.
 """
@@ -37,7 +38,7 @@ class HotPath:
                  order: int = vpic.VPIC_SORT_STANDARD, math: int = vpic.MATH_FAST,
                  deposit: int = vpic.DEP_AUTO, tile_sz: int = 0, rank: int = 0, nranks: int = 1,
                  uid: bytes = None, capacity_factor: float = 1.0, max_movers: int = 1 << 20,
-                 device: Optional[int] = None):
+                 device: Optional[int] = None, field_solve: bool = False, eps0: float = 1.0):
         vpic.load()
         self.wl = wl
         self.g = wl.grid
@@ -47,6 +48,8 @@ class HotPath:
         self.ctx.set_option(vpic.VPIC_OPT_DEPOSIT, deposit)
         self.order = order
         self.tile_sz = tile_sz
+        self.field_solve = field_solve   # advance_b(1/2), advance_e, advance_b(1/2) after unload
+        self.eps0 = eps0
         self.nranks = nranks
         self.migrate = nranks > 1 or any(b == inputs.BC_ABSORB for b in self.g.pbc)
         nv = self.g.nv
@@ -107,6 +110,10 @@ class HotPath:
                                                    s.movers, s.n_movers, self.acc)
                 s.n_movers.zero_()
         vpic.vpic_unload_accumulator(self.ctx, self.acc, self.jf)
+        if self.field_solve:
+            vpic.vpic_advance_b(self.ctx, self.fields, 0.5)
+            vpic.vpic_advance_e(self.ctx, self.fields, self.jf, self.eps0)
+            vpic.vpic_advance_b(self.ctx, self.fields, 0.5)
 
     def cycle(self, steps: int):
         """One sort period: sort, then `steps` PIC steps."""

@@ -1,0 +1,84 @@
+"""GPU parity of the field solver (vpic_advance_b / vpic_advance_e, §8(f) f1)
+and of a self-consistent PIC step (push -> unload -> field advance).
+
+The Yee updates use the oracle's expressions in the same order without FMA,
+so fields are bit-exact given identical inputs; through a full step the only
+difference is jf (float atomics reordered), bounded by T1.
+"""
+import numpy as np
+import pytest
+import torch
+
+from paper_conf_sc_tanlta25_b200 import inputs
+from parity_util import assert_particles_bitexact
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def V():
+    from paper_conf_sc_tanlta25_b200 import _build, vpic
+    _build.build()
+    vpic.load()
+    return vpic
+
+
+GRIDS = [inputs.GridSpec(9, 6, 5, dx=0.7, dy=1.0, dz=1.3, dt=0.4),
+         inputs.GridSpec(16, 16, 16),
+         inputs.GridSpec(7, 5, 4, pbc=(0, 0, 1, 0, 0, 1))]
+
+
+@pytest.mark.parametrize("g", GRIDS, ids=["noncubic", "cube16", "reflect_z"])
+def test_advance_b_e_bitexact(V, orc, g):
+    rng = np.random.default_rng(4)
+    f = rng.standard_normal((g.nv, 8)).astype(np.float32)
+    f[:, 3] = 0
+    f[:, 7] = 0
+    jf = rng.standard_normal((g.nv, 4)).astype(np.float32)
+    ctx = V.Context(g)
+    fd = torch.from_numpy(f.copy()).cuda()
+    jd = torch.from_numpy(jf).cuda()
+    fo = f.copy()
+    for frac in (0.5, 0.25, 1.0):
+        V.vpic_advance_b(ctx, fd, frac)
+        orc.advance_b(g, fo, frac)
+        V.vpic_advance_e(ctx, fd, jd, 1.3)
+        orc.advance_e(g, fo, jf, 1.3)
+    torch.cuda.synchronize()
+    got = fd.cpu().numpy()
+    assert np.array_equal(got.view(np.uint32), fo.view(np.uint32))
+
+
+def test_pic_step_with_field_solve(V, orc):
+    """Two self-consistent steps (IEEE math): after step 1 the particles are
+    bit-exact and the fields within the jf tolerance; step 2 pushes with those
+    fields and stays within the FAST-mode tolerances."""
+    from paper_conf_sc_tanlta25_b200.pic import HotPath
+    wl = inputs.config(0)
+    g = wl.grid
+    parts = inputs.make_species_particles(wl)
+    fields = inputs.make_fields(g, 0.05)
+    hp = HotPath(wl, parts, fields, math=V.MATH_IEEE, field_solve=True)
+    hp.step(do_sort=False)
+    torch.cuda.synchronize()
+    # oracle step
+    fo = fields.copy()
+    interp = orc.load_interpolator(g, fo)
+    acc = np.zeros((g.nv, 12), np.float32)
+    aabs = np.zeros((g.nv, 12), np.float64)
+    po = [p.copy() for p in parts]
+    for sp, p in zip(wl.species, po):
+        orc.advance_p(g, sp.q, sp.m, p, interp, acc, aabs)
+    jf = orc.unload_accumulator(g, acc)
+    jfabs = orc.unload_accumulator(g, np.abs(acc)).astype(np.float64)
+    orc.advance_b(g, fo, 0.5)
+    orc.advance_e(g, fo, jf, 1.0)
+    orc.advance_b(g, fo, 0.5)
+    for k in range(2):
+        assert_particles_bitexact(hp.particles_host(k), po[k])
+    got = hp.fields.cpu().numpy().astype(np.float64)
+    cj = g.dt / 1.0
+    # E carries -cj * jf (jf within 1e-5 of its abs-sum); cB sees it through curl E
+    tol = 1e-5 * cj * jfabs.max() * 4 + 1e-6 * np.abs(fo).max()
+    vox = g.interior_voxels()
+    assert np.abs(got[vox] - fo[vox].astype(np.float64)).max() <= tol

@@ -49,6 +49,8 @@ def parse():
     ap.add_argument("--math", default="fast", choices=["fast", "ieee"])
     ap.add_argument("--deposit", default="auto", choices=["auto", "lane", "warp"])
     ap.add_argument("--kernel", default="auto", choices=["auto", "direct", "tma"])
+    ap.add_argument("--field-solve", action="store_true",
+                    help="full PIC step: + advance_b/advance_e (self-consistent fields)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no e2e/cpu legs)")
@@ -235,7 +237,8 @@ def our_arm(args, rank, world):
     dep = {"auto": 0, "lane": 1, "warp": 2}[args.deposit]
     cap = 1.0 if world == 1 else 1.05
     hp = HotPath(wl, parts, fields, order=order, math=math_mode, deposit=dep, rank=rank,
-                 nranks=world, uid=uid, capacity_factor=cap, device=local)
+                 nranks=world, uid=uid, capacity_factor=cap, device=local,
+                 field_solve=args.field_solve)
     hp.ctx.set_option(vpic.VPIC_OPT_ADVANCE_KERNEL, {"auto": 0, "direct": 1, "tma": 2}[args.kernel])
     n_local = hp.n_particles
 
@@ -332,6 +335,7 @@ def our_arm(args, rank, world):
                    "species": len(wl.species), "particles": int(ntot), "sort_every": S,
                    "order": args.order, "shuffled": bool(args.shuffle), "math": args.math,
                    "deposit": args.deposit, "kernel": args.kernel, "parallelism": f"domain{world}",
+                   "field_solve": bool(args.field_solve),
                    "l2": f"no flush: inputs ({32 * n_local / 1e9:.1f} GB of particles per GPU) >> 126 MB L2"},
         "per_gpu": value / world,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",

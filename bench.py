@@ -51,6 +51,8 @@ def parse():
     ap.add_argument("--kernel", default="auto", choices=["auto", "direct", "tma"])
     ap.add_argument("--field-solve", action="store_true",
                     help="full PIC step: + advance_b/advance_e (self-consistent fields)")
+    ap.add_argument("--loopback", action="store_true",
+                    help="1 GPU: periodic faces through the NCCL exchange (self peer)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no e2e/cpu legs)")
@@ -238,7 +240,7 @@ def our_arm(args, rank, world):
     cap = 1.0 if world == 1 else 1.05
     hp = HotPath(wl, parts, fields, order=order, math=math_mode, deposit=dep, rank=rank,
                  nranks=world, uid=uid, capacity_factor=cap, device=local,
-                 field_solve=args.field_solve)
+                 field_solve=args.field_solve, loopback_exchange=args.loopback and world == 1)
     hp.ctx.set_option(vpic.VPIC_OPT_ADVANCE_KERNEL, {"auto": 0, "direct": 1, "tma": 2}[args.kernel])
     n_local = hp.n_particles
 
@@ -334,7 +336,8 @@ def our_arm(args, rank, world):
         "config": {"workload": wl.name, "cells_per_gpu": [g.nx, g.ny, g.nz], "ppc_per_species": wl.ppc,
                    "species": len(wl.species), "particles": int(ntot), "sort_every": S,
                    "order": args.order, "shuffled": bool(args.shuffle), "math": args.math,
-                   "deposit": args.deposit, "kernel": args.kernel, "parallelism": f"domain{world}",
+                   "deposit": args.deposit, "kernel": args.kernel,
+                   "parallelism": "loopback1" if args.loopback and world == 1 else f"domain{world}",
                    "field_solve": bool(args.field_solve),
                    "l2": f"no flush: inputs ({32 * n_local / 1e9:.1f} GB of particles per GPU) >> 126 MB L2"},
         "per_gpu": value / world,

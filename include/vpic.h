@@ -80,7 +80,13 @@ enum {
   VPIC_OPT_TILE_SZ = 2,
   /* advance_p kernel variant: 0 = AUTO, 1 = direct global loads,
    * 2 = TMA bulk-copy pipeline (particles staged through shared memory). */
-  VPIC_OPT_ADVANCE_KERNEL = 3
+  VPIC_OPT_ADVANCE_KERNEL = 3,
+  /* 1 = route every PERIODIC face of a single-rank context through the NCCL
+   * exchange with the rank itself as the peer (a one-rank communicator):
+   * particle migration, E/cB halos and the jf plane reduction then run the
+   * multi-GPU code path on one GPU, and must reproduce the local periodic
+   * wrap.  Validation of the exchange; set once, before any other call. */
+  VPIC_OPT_LOOPBACK_EXCHANGE = 4
 };
 
 typedef struct {

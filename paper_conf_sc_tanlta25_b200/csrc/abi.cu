@@ -176,6 +176,19 @@ int vpic_ctx_set_option(vpic_ctx *c, int option, int64_t value) {
       if (value < ADV_AUTO || value > ADV_TMA) return VPIC_ERR_INVALID;
       c->adv_kernel = (int)value;
       return VPIC_OK;
+    case VPIC_OPT_LOOPBACK_EXCHANGE: {
+      if (value != 1 || c->nranks != 1 || c->ex) return VPIC_ERR_INVALID;
+      DeviceGuard dg(c->device);
+      uint8_t uid[128];
+      int rc = vpic_get_unique_id(uid);
+      if (rc != VPIC_OK) return rc;
+      rc = exchange_create(c, uid);
+      if (rc != VPIC_OK) return rc;
+      for (int f = 0; f < 6; ++f)
+        if (c->g.pbc[f] == VPIC_BC_PERIODIC) c->gk.face_kind[f] = FACE_REMOTE;
+      for (int a = 0; a < 3; ++a) c->periodic_local[a] = false;
+      return VPIC_OK;
+    }
     default:
       return VPIC_ERR_INVALID;
   }

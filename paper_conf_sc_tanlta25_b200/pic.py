@@ -38,7 +38,8 @@ class HotPath:
                  order: int = vpic.VPIC_SORT_STANDARD, math: int = vpic.MATH_FAST,
                  deposit: int = vpic.DEP_AUTO, tile_sz: int = 0, rank: int = 0, nranks: int = 1,
                  uid: bytes = None, capacity_factor: float = 1.0, max_movers: int = 1 << 20,
-                 device: Optional[int] = None, field_solve: bool = False, eps0: float = 1.0):
+                 device: Optional[int] = None, field_solve: bool = False, eps0: float = 1.0,
+                 loopback_exchange: bool = False):
         vpic.load()
         self.wl = wl
         self.g = wl.grid
@@ -51,7 +52,10 @@ class HotPath:
         self.field_solve = field_solve   # advance_b(1/2), advance_e, advance_b(1/2) after unload
         self.eps0 = eps0
         self.nranks = nranks
-        self.migrate = nranks > 1 or any(b == inputs.BC_ABSORB for b in self.g.pbc)
+        if loopback_exchange:   # periodic faces through the NCCL path (self peer)
+            self.ctx.set_option(vpic.VPIC_OPT_LOOPBACK_EXCHANGE, 1)
+        self.migrate = (nranks > 1 or loopback_exchange
+                        or any(b == inputs.BC_ABSORB for b in self.g.pbc))
         nv = self.g.nv
         f32 = dict(dtype=torch.float32, device=self.dev)
         self.fields = torch.from_numpy(np.ascontiguousarray(fields)).to(self.dev)

@@ -40,9 +40,11 @@ struct Ptrs6 { float4 *p[6]; };
 // (remote face: packed for the neighbour with its entry voxel and flipped
 // offset; absorb face: dropped).  Its slot becomes a hole.
 __global__ void k_pack_movers(const GridK g, const vpic_particle_t *__restrict__ p,
-                              const vpic_mover_t *__restrict__ mv, int64_t M, float4 *__restrict__ send,
+                              const vpic_mover_t *__restrict__ mv, const int64_t *__restrict__ Mdev,
+                              int64_t Mmax, float4 *__restrict__ send,
                               int64_t send_cap, int64_t *__restrict__ send_cnt,
                               uint32_t *__restrict__ holes, int32_t *__restrict__ flags) {
+  const int64_t M = min(*Mdev, Mmax);
   for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < M;
        k += (int64_t)gridDim.x * blockDim.x) {
     const vpic_mover_t m = mv[k];
@@ -86,7 +88,9 @@ __global__ void k_tail_survivors(const uint32_t *__restrict__ tail_dead, int64_t
     if (!tail_dead[j]) surv[atomicAdd(nsurv, 1ull)] = (uint32_t)(np_new + j);
 }
 __global__ void k_backfill(vpic_particle_t *__restrict__ p, const uint32_t *__restrict__ low,
-                           const uint32_t *__restrict__ surv, int64_t n) {
+                           const uint32_t *__restrict__ surv,
+                           const unsigned long long *__restrict__ nlow) {
+  const int64_t n = (int64_t)*nlow;
   for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n;
        k += (int64_t)gridDim.x * blockDim.x)
     p[low[k]] = p[surv[k]];
@@ -173,15 +177,13 @@ int remove_holes(vpic_ctx *c, vpic_particle_t *p, int64_t np, const uint32_t *ho
   const int64_t np_new = np - H;
   uint32_t *sc = static_cast<uint32_t *>(c->scratch) + H;  // after the hole list
   uint32_t *tail_dead = sc, *low = sc + H, *surv = sc + 2 * H;
-  unsigned long long *cnt = reinterpret_cast<unsigned long long *>(c->d_count + 2);
+  unsigned long long *cnt = reinterpret_cast<unsigned long long *>(c->d_count + 4);  // [4], [5]
   CKC(cudaMemsetAsync(tail_dead, 0, 4 * (size_t)H, s));
   CKC(cudaMemsetAsync(cnt, 0, 16, s));
   k_mark_tail<<<blocks_for(H), 256, 0, s>>>(holes, H, np_new, tail_dead, low, cnt); note_launch();
   k_tail_survivors<<<blocks_for(H), 256, 0, s>>>(tail_dead, H, np_new, surv, cnt + 1); note_launch();
-  int64_t h_low = 0;
-  CKC(cudaMemcpyAsync(&h_low, cnt, 8, cudaMemcpyDeviceToHost, s));
-  CKC(cudaStreamSynchronize(s));
-  if (h_low) { k_backfill<<<blocks_for(h_low), 256, 0, s>>>(p, low, surv, h_low); note_launch(); }
+  // as many tail survivors as holes below np_new: the device count sizes it
+  k_backfill<<<blocks_for(H), 256, 0, s>>>(p, low, surv, cnt); note_launch();
   return cudaGetLastError() == cudaSuccess ? VPIC_OK : VPIC_ERR_CUDA;
 }
 
@@ -222,6 +224,8 @@ void exchange_destroy(vpic_ctx *c) {
 
 // Up to 3 rounds: pack movers per face, exchange counts, exchange records,
 // remove departed / absorbed particles, append arrivals, continue their move.
+// Host synchronisations: the initial mover count, one per round (the NCCL
+// record sizes, which also return the round's mover count), one for flags.
 int migrate(vpic_ctx *c, float qsp, float msp, vpic_particle_t *p, int64_t *np_io, int64_t max_np,
             vpic_mover_t *movers, const int64_t *n_movers, float *acc, cudaStream_t s) {
   (void)msp;
@@ -234,11 +238,13 @@ int migrate(vpic_ctx *c, float qsp, float msp, vpic_particle_t *p, int64_t *np_i
   CKC(cudaMemsetAsync(d_flags, 0, 4, s));
   Exchange *ex = c->ex;
   const vpic_mover_t *cur = movers;
+  const int64_t *Mdev = n_movers;   // device count of the current mover list
+  int64_t Mmax = M;                 // host upper bound of it
   const int rounds = ex ? 3 : 1;
   for (int round = 0; round <= rounds; ++round) {
     const bool exchange = ex && round < rounds;
-    if (!exchange && M == 0) break;
-    const int64_t Mpad = std::max<int64_t>(M, 1);
+    if (!exchange && Mmax == 0) break;
+    const int64_t Mpad = std::max<int64_t>(Mmax, 1);
     if (int rc = ctx_scratch(c, 16 * (size_t)Mpad + 64)) return rc;
     uint32_t *holes = static_cast<uint32_t *>(c->scratch);
     int64_t *cnt = ex ? ex->d_cnt : c->d_count + 3;
@@ -248,9 +254,9 @@ int migrate(vpic_ctx *c, float qsp, float msp, vpic_particle_t *p, int64_t *np_i
       ex->send_cap = tot / 6;
     }
     CKC(cudaMemsetAsync(cnt, 0, (ex ? 12 : 1) * sizeof(int64_t), s));
-    if (M > 0) {
-      k_pack_movers<<<blocks_for(M), 256, 0, s>>>(c->gk, p, cur, M, exchange ? ex->send : nullptr,
-                                                   exchange ? ex->send_cap : 0, cnt, holes, d_flags); note_launch();
+    if (Mmax > 0) {
+      k_pack_movers<<<blocks_for(Mmax), 256, 0, s>>>(c->gk, p, cur, Mdev, Mmax, exchange ? ex->send : nullptr,
+                                                      exchange ? ex->send_cap : 0, cnt, holes, d_flags); note_launch();
       CKC(cudaGetLastError());
     }
     int64_t sent[6] = {0, 0, 0, 0, 0, 0}, rcvd[6] = {0, 0, 0, 0, 0, 0}, A = 0;
@@ -267,9 +273,11 @@ int migrate(vpic_ctx *c, float qsp, float msp, vpic_particle_t *p, int64_t *np_i
           CKN(ncclRecv(cnt + 6 + o, 1, ncclInt64, c->g.nbr_rank[o], ex->comm, s));
       }
       CKN(ncclGroupEnd());
-      int64_t h[12];
-      CKC(cudaMemcpyAsync(h, cnt, sizeof(h), cudaMemcpyDeviceToHost, s));
+      int64_t h[13];
+      CKC(cudaMemcpyAsync(h, cnt, 12 * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+      CKC(cudaMemcpyAsync(h + 12, Mdev, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
       CKC(cudaStreamSynchronize(s));
+      M = std::min(h[12], Mmax);
       for (int f = 0; f < 6; ++f) {
         sent[f] = h[f];
         rcvd[f] = h[6 + f];
@@ -292,13 +300,17 @@ int migrate(vpic_ctx *c, float qsp, float msp, vpic_particle_t *p, int64_t *np_i
           CKN(ncclRecv(rptr[o], (size_t)rcvd[o] * 12, ncclFloat32, c->g.nbr_rank[o], ex->comm, s));
       }
       CKN(ncclGroupEnd());
+    } else if (round > 0) {  // final clean-up round: the exact count of the leftovers
+      CKC(cudaMemcpyAsync(&M, Mdev, 8, cudaMemcpyDeviceToHost, s));
+      CKC(cudaStreamSynchronize(s));
+      M = std::min(M, Mmax);
     }
     // every mover's particle has left this rank (sent or absorbed)
     if (int rc = remove_holes(c, p, np, holes, M, s)) return rc;
     np -= M;
-    M = 0;
     if (!exchange) break;
     if (np + A > max_np) return VPIC_ERR_CAPACITY;
+    Mmax = 0;
     if (A > 0) {
       if (int rc = ensure(reinterpret_cast<void **>(&ex->mv_arr), &ex->mv_arr_cap, A, 16)) return rc;
       if (int rc = ensure(reinterpret_cast<void **>(&ex->mv_next), &ex->mv_next_cap, A, 16)) return rc;
@@ -310,10 +322,10 @@ int migrate(vpic_ctx *c, float qsp, float msp, vpic_particle_t *p, int64_t *np_i
                           ? launch_move_movers_ieee(c, qsp, p, ex->mv_arr, A, acc, ex->mv_next, A, d_next, d_flags, s)
                           : launch_move_movers_fast(c, qsp, p, ex->mv_arr, A, acc, ex->mv_next, A, d_next, d_flags, s);
       CKC(e);
-      CKC(cudaMemcpyAsync(&M, d_next, 8, cudaMemcpyDeviceToHost, s));
-      CKC(cudaStreamSynchronize(s));
       np += A;
       cur = ex->mv_next;
+      Mdev = d_next;
+      Mmax = A;     // the arrivals' new movers: at most A, exact count on device
     }
   }
   int32_t hflag = 0;

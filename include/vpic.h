@@ -204,6 +204,22 @@ int vpic_unload_accumulator(vpic_ctx *ctx, const float *acc, float *jf, void *st
 int vpic_advance_b(vpic_ctx *ctx, float *fields, float frac, void *stream);
 int vpic_advance_e(vpic_ctx *ctx, float *fields, const float *jf, float eps0, void *stream);
 
+/* ---------------------------- (f2) gather-scatter microbenchmark kernel -- */
+
+/* The gather-scatter kernel of the paper's sorting study ("one billion
+ * double-precision numbers using three key patterns ... Memory bandwidth is
+ * calculated based on the total amount of data movement").  For
+ * each i < n with k = keys[i] (0 <= k < nkeys), the access set is {k}
+ * (stencil_nx == 0) or the 5-point stencil {k, k-1, k+1, k-nx, k+nx} (mod
+ * nkeys, reading F2); out[i] = sum of table[] over the set, and x[i] is added
+ * to acc[] at every point of the set (aggregate = 0: one red.global.add.f64
+ * per lane and point -- the paper's atomic scatter; 1: lanes of a warp that
+ * share a point are summed first).  keys[n] int32, x/out[n], table/acc[nkeys]
+ * float64, all device memory. */
+int vpic_gather_scatter(vpic_ctx *ctx, const int32_t *keys, const double *x, int64_t n,
+                        const double *table, double *out, double *acc, int64_t nkeys,
+                        int64_t stencil_nx, int aggregate, void *stream);
+
 /* ---------------------------------------------------- (a13) exchange -- */
 
 /* Finish the movers produced by vpic_advance_p for one species: particles on

@@ -80,6 +80,8 @@ def lib() -> ctypes.CDLL:
         _lib.orc_advance_b.restype = None
         _lib.orc_advance_e.argtypes = [G, P, P, ctypes.c_float]
         _lib.orc_advance_e.restype = None
+        _lib.orc_gather_scatter.argtypes = [P, P, I64, P, P, P, I64, I64]
+        _lib.orc_gather_scatter.restype = None
     return _lib
 
 
@@ -203,3 +205,15 @@ def advance_e(spec, fields, jf, eps0=1.0):
     jf = np.ascontiguousarray(jf, dtype=np.float32)
     g = make_grid(spec)
     lib().orc_advance_e(ctypes.byref(g), _ptr(fields), _ptr(jf), eps0)
+
+
+# ------------------------------------------------------ gather-scatter (f2) --
+def gather_scatter(keys, x, table, acc, stencil_nx=0):
+    """Returns out[n]; acc (float64[nkeys]) updated in place."""
+    keys = np.ascontiguousarray(keys, dtype=np.int32)
+    x = np.ascontiguousarray(x, dtype=np.float64)
+    table = np.ascontiguousarray(table, dtype=np.float64)
+    out = np.empty(keys.size, np.float64)
+    lib().orc_gather_scatter(_ptr(keys), _ptr(x), keys.size, _ptr(table), _ptr(out), _ptr(acc),
+                             table.size, stencil_nx)
+    return out

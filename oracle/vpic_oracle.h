@@ -97,6 +97,13 @@ int64_t orc_remove_absorbed(const orc_grid *g, orc_particle *p, int64_t np,
 void orc_advance_b(const orc_grid *g, float *fields, float frac);
 void orc_advance_e(const orc_grid *g, float *fields, const float *jf, float eps0);
 
+/* Gather-scatter microbenchmark of PAPER.md:236-242 (f2, reading F2): for
+ * each i, the access set is {k} (stencil_nx == 0) or {k, k-1, k+1, k-nx,
+ * k+nx} (mod nkeys), k = keys[i]; out[i] = sum of table over the set (in that
+ * order) and acc[k'] += x[i] for every k' of the set.  FP64, serial. */
+void orc_gather_scatter(const int32_t *keys, const double *x, int64_t n, const double *table,
+                        double *out, double *acc, int64_t nkeys, int64_t stencil_nx);
+
 #ifdef __cplusplus
 }
 #endif

@@ -45,6 +45,7 @@ def _units():
         ("grid_ops.o", "grid_ops.cu", ["-fmad=false"]),
         ("sort.o", "sort.cu", []),
         ("migrate.o", "migrate.cu", []),
+        ("gather_scatter.o", "gather_scatter.cu", []),
         ("abi.o", "abi.cu", []),
     ], I
 

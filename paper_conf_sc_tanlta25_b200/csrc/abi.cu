@@ -293,6 +293,16 @@ int vpic_advance_e(vpic_ctx *c, float *fields, const float *jf, float eps0, void
   return cuda_status(launch_advance_e(c, fields, jf, eps0, S(stream)));
 }
 
+int vpic_gather_scatter(vpic_ctx *c, const int32_t *keys, const double *x, int64_t n,
+                        const double *table, double *out, double *acc, int64_t nkeys,
+                        int64_t stencil_nx, int aggregate, void *stream) {
+  if (!c || n < 0 || nkeys <= 0 || nkeys >= ((int64_t)1 << 31) || stencil_nx < 0) return VPIC_ERR_INVALID;
+  if (n > 0 && (!keys || !x || !table || !out || !acc)) return VPIC_ERR_INVALID;
+  DeviceGuard dg(c->device);
+  return cuda_status(launch_gather_scatter(c, keys, x, n, table, out, acc, nkeys, stencil_nx,
+                                           aggregate, S(stream)));
+}
+
 int vpic_migrate_particles(vpic_ctx *c, float q, float m, vpic_particle_t *p, int64_t *np,
                            int64_t max_np, vpic_mover_t *movers, const int64_t *n_movers,
                            float *acc, void *stream) {

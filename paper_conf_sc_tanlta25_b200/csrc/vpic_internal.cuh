@@ -85,6 +85,10 @@ cudaError_t launch_advance_b(const vpic_ctx *c, float *fields, float frac, cudaS
 cudaError_t launch_advance_e(const vpic_ctx *c, float *fields, const float *jf, float eps0,
                              cudaStream_t s);
 
+cudaError_t launch_gather_scatter(const vpic_ctx *c, const int32_t *keys, const double *x,
+                                  int64_t n, const double *table, double *out, double *acc,
+                                  int64_t nkeys, int64_t nx, int aggregate, cudaStream_t s);
+
 size_t sort_workspace_bytes(const vpic_ctx *c, int64_t np, int order);
 cudaError_t launch_sort(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_t *p_out,
                         int64_t np, int order, int64_t tile_sz, void *ws, size_t ws_bytes,

@@ -31,7 +31,7 @@ EXPORTS = ["vpic_get_unique_id", "vpic_ctx_create", "vpic_ctx_destroy", "vpic_ct
            "vpic_ctx_info", "vpic_status_string", "vpic_sort_workspace_bytes",
            "vpic_sort_particles", "vpic_load_interpolator", "vpic_clear_accumulator",
            "vpic_advance_p", "vpic_unload_accumulator", "vpic_migrate_particles",
-           "vpic_kernel_launches", "vpic_advance_b", "vpic_advance_e"]
+           "vpic_kernel_launches", "vpic_advance_b", "vpic_advance_e", "vpic_gather_scatter"]
 
 
 class VpicError(RuntimeError):
@@ -76,6 +76,7 @@ def load(path: str = LIB_PATH) -> ctypes.CDLL:
         "vpic_advance_p": ([P, ctypes.c_float, ctypes.c_float, P, I64, P, P, P, I64, P, P, P], I),
         "vpic_unload_accumulator": ([P, P, P, P], I),
         "vpic_advance_b": ([P, P, ctypes.c_float, P], I),
+        "vpic_gather_scatter": ([P, P, P, I64, P, P, P, I64, I64, I, P], I),
         "vpic_advance_e": ([P, P, P, ctypes.c_float, P], I),
         "vpic_migrate_particles": ([P, ctypes.c_float, ctypes.c_float, P, ctypes.POINTER(I64),
                                     I64, P, P, P, P], I),
@@ -213,6 +214,13 @@ def vpic_advance_b(ctx: Context, fields, frac: float, stream=None):
 def vpic_advance_e(ctx: Context, fields, jf, eps0: float = 1.0, stream=None):
     _check("vpic_advance_e", load().vpic_advance_e(ctx.h, _ptr(fields), _ptr(jf), eps0,
                                                    _stream(stream)))
+
+
+def vpic_gather_scatter(ctx: Context, keys, x, table, out, acc, stencil_nx: int = 0,
+                        aggregate: int = 0, stream=None):
+    _check("vpic_gather_scatter", load().vpic_gather_scatter(
+        ctx.h, _ptr(keys), _ptr(x), keys.numel(), _ptr(table), _ptr(out), _ptr(acc), table.numel(),
+        stencil_nx, aggregate, _stream(stream)))
 
 
 def vpic_migrate_particles(ctx: Context, q: float, m: float, p, np_: int, max_np: int, movers,

@@ -296,3 +296,32 @@ def test_run_host_cycles_matches_device_cycles(V):
         got = host_out[k].numpy().view(inputs.PARTICLE_DTYPE).reshape(-1)
         assert_particles_bitexact(got, want[k])
     assert np.all(np.isfinite(jf_host.numpy()))
+
+
+@pytest.mark.parametrize("nx", [0, 37])
+@pytest.mark.parametrize("agg", [0, 1])
+@pytest.mark.parametrize("order", ["sorted", "strided", "random"])
+def test_gather_scatter_parity(V, orc, nx, agg, order):
+    rng = np.random.default_rng(5)
+    K, m = 3001, 70
+    if order == "sorted":
+        keys = np.repeat(np.arange(K), m)
+    elif order == "strided":
+        keys = np.tile(np.arange(K), m)
+    else:
+        keys = rng.permutation(np.repeat(np.arange(K), m))
+    keys = keys.astype(np.int32)
+    x = rng.standard_normal(keys.size)
+    table = rng.standard_normal(K)
+    acc_o = np.zeros(K)
+    out_o = orc.gather_scatter(keys, x, table, acc_o, nx)
+    ctx = mkctx(V, inputs.GridSpec(4, 4, 4))
+    kd, xd, td = (torch.from_numpy(a).cuda() for a in (keys, x, table))
+    out = torch.empty_like(xd)
+    acc = torch.zeros(K, dtype=torch.float64, device="cuda")
+    V.vpic_gather_scatter(ctx, kd, xd, td, out, acc, nx, agg)
+    torch.cuda.synchronize()
+    assert np.array_equal(out.cpu().numpy(), out_o)               # same summation order
+    absum = np.zeros(K)
+    orc.gather_scatter(keys, np.abs(x), table, absum, nx)
+    assert np.all(np.abs(acc.cpu().numpy() - acc_o) <= 1e-13 * absum + 1e-300)

@@ -220,6 +220,29 @@ int vpic_gather_scatter(vpic_ctx *ctx, const int32_t *keys, const double *x, int
                         const double *table, double *out, double *acc, int64_t nkeys,
                         int64_t stencil_nx, int aggregate, void *stream);
 
+/* ------------------------- (f4) on-line charge-conservation diagnostics -- */
+
+/* Cloud-in-cell charge on the nodes (VPIC accumulate_rho_p, ref. [3]; reading
+ * D1): for each particle, rho[node] += q w (1 +- dx)(1 +- dy)(1 +- dz) / 8 on
+ * the 8 nodes (x..x+1, y..y+1, z..z+1) of its voxel, the sign of each factor
+ * set by the side of the node.  Node n+1 of a locally periodic axis is node 1;
+ * other n+1 nodes are kept (a REMOTE face's shared nodes are NOT summed with
+ * the neighbour: single-rank diagnostic).  rho[nv] float32 device memory
+ * indexed like voxels, ACCUMULATED into.  np == 0 is a no-op. */
+int vpic_accumulate_rho(vpic_ctx *ctx, float q, const vpic_particle_t *p, int64_t np, float *rho,
+                        void *stream);
+
+/* Discrete continuity residual of the charge-conserving deposit ("the
+ * discrete continuity invariant", BASELINE north_star; deposit P:238):
+ *   res(node) = (rho1 - rho0) / (dx dy dz dt) + sum_a (jf_a(node) - jf_a(node - e_a)) / d_a
+ * over the nodes 1..n of a locally periodic axis (node - e_a wraps to n) and
+ * 1..n+1 otherwise.  rho0/rho1 from vpic_accumulate_rho before/after one
+ * vpic_advance_p of every species, jf from vpic_unload_accumulator.
+ *   out  device float[2], overwritten: {max |res|, max |drho/dt|};
+ *   res  device float[nv] (nullable): res per node, other entries untouched. */
+int vpic_continuity_residual(vpic_ctx *ctx, const float *rho0, const float *rho1, const float *jf,
+                             float *out, float *res, void *stream);
+
 /* ---------------------------------------------------- (a13) exchange -- */
 
 /* Finish the movers produced by vpic_advance_p for one species: particles on

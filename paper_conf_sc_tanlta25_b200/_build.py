@@ -46,6 +46,7 @@ def _units():
         ("sort.o", "sort.cu", []),
         ("migrate.o", "migrate.cu", []),
         ("gather_scatter.o", "gather_scatter.cu", []),
+        ("diagnostics.o", "diagnostics.cu", ["-fmad=false"]),
         ("abi.o", "abi.cu", []),
     ], I
 

@@ -293,6 +293,20 @@ int vpic_advance_e(vpic_ctx *c, float *fields, const float *jf, float eps0, void
   return cuda_status(launch_advance_e(c, fields, jf, eps0, S(stream)));
 }
 
+int vpic_accumulate_rho(vpic_ctx *c, float q, const vpic_particle_t *p, int64_t np, float *rho,
+                        void *stream) {
+  if (!c || np < 0 || !rho || (np > 0 && (!p || !aligned16(p)))) return VPIC_ERR_INVALID;
+  DeviceGuard dg(c->device);
+  return cuda_status(launch_accumulate_rho(c, q, p, np, rho, S(stream)));
+}
+
+int vpic_continuity_residual(vpic_ctx *c, const float *rho0, const float *rho1, const float *jf,
+                             float *out, float *res, void *stream) {
+  if (!c || !rho0 || !rho1 || !jf || !out || !aligned16(jf)) return VPIC_ERR_INVALID;
+  DeviceGuard dg(c->device);
+  return cuda_status(launch_continuity(c, rho0, rho1, jf, out, res, S(stream)));
+}
+
 int vpic_gather_scatter(vpic_ctx *c, const int32_t *keys, const double *x, int64_t n,
                         const double *table, double *out, double *acc, int64_t nkeys,
                         int64_t stencil_nx, int aggregate, void *stream) {

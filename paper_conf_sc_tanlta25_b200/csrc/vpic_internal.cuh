@@ -85,6 +85,10 @@ cudaError_t launch_advance_b(const vpic_ctx *c, float *fields, float frac, cudaS
 cudaError_t launch_advance_e(const vpic_ctx *c, float *fields, const float *jf, float eps0,
                              cudaStream_t s);
 
+cudaError_t launch_accumulate_rho(const vpic_ctx *c, float q, const vpic_particle_t *p, int64_t np,
+                                  float *rho, cudaStream_t s);
+cudaError_t launch_continuity(const vpic_ctx *c, const float *rho0, const float *rho1,
+                              const float *jf, float *out, float *res, cudaStream_t s);
 cudaError_t launch_gather_scatter(const vpic_ctx *c, const int32_t *keys, const double *x,
                                   int64_t n, const double *table, double *out, double *acc,
                                   int64_t nkeys, int64_t nx, int aggregate, cudaStream_t s);

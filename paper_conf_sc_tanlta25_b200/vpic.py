@@ -16,7 +16,7 @@ import torch
 from .inputs import GridSpec
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libvpic.so")
+LIB_PATH = os.environ.get("VPIC_LIB") or os.path.join(_HERE, "libvpic.so")  # VPIC_LIB: dev A/B builds
 
 VPIC_OK, VPIC_ERR_INVALID, VPIC_ERR_CAPACITY = 0, -1, -2
 VPIC_ERR_CUDA, VPIC_ERR_NCCL, VPIC_ERR_UNSUPPORTED = -3, -4, -5
@@ -31,7 +31,8 @@ EXPORTS = ["vpic_get_unique_id", "vpic_ctx_create", "vpic_ctx_destroy", "vpic_ct
            "vpic_ctx_info", "vpic_status_string", "vpic_sort_workspace_bytes",
            "vpic_sort_particles", "vpic_load_interpolator", "vpic_clear_accumulator",
            "vpic_advance_p", "vpic_unload_accumulator", "vpic_migrate_particles",
-           "vpic_kernel_launches", "vpic_advance_b", "vpic_advance_e", "vpic_gather_scatter"]
+           "vpic_kernel_launches", "vpic_advance_b", "vpic_advance_e", "vpic_gather_scatter",
+           "vpic_accumulate_rho", "vpic_continuity_residual"]
 
 
 class VpicError(RuntimeError):
@@ -77,6 +78,8 @@ def load(path: str = LIB_PATH) -> ctypes.CDLL:
         "vpic_unload_accumulator": ([P, P, P, P], I),
         "vpic_advance_b": ([P, P, ctypes.c_float, P], I),
         "vpic_gather_scatter": ([P, P, P, I64, P, P, P, I64, I64, I, P], I),
+        "vpic_accumulate_rho": ([P, ctypes.c_float, P, I64, P, P], I),
+        "vpic_continuity_residual": ([P, P, P, P, P, P, P], I),
         "vpic_advance_e": ([P, P, P, ctypes.c_float, P], I),
         "vpic_migrate_particles": ([P, ctypes.c_float, ctypes.c_float, P, ctypes.POINTER(I64),
                                     I64, P, P, P, P], I),
@@ -221,6 +224,17 @@ def vpic_gather_scatter(ctx: Context, keys, x, table, out, acc, stencil_nx: int 
     _check("vpic_gather_scatter", load().vpic_gather_scatter(
         ctx.h, _ptr(keys), _ptr(x), keys.numel(), _ptr(table), _ptr(out), _ptr(acc), table.numel(),
         stencil_nx, aggregate, _stream(stream)))
+
+
+def vpic_accumulate_rho(ctx: Context, q: float, p, np_: int, rho, stream=None):
+    _check("vpic_accumulate_rho", load().vpic_accumulate_rho(ctx.h, q, _ptr(p), np_, _ptr(rho),
+                                                             _stream(stream)))
+
+
+def vpic_continuity_residual(ctx: Context, rho0, rho1, jf, out, res=None, stream=None):
+    _check("vpic_continuity_residual", load().vpic_continuity_residual(
+        ctx.h, _ptr(rho0), _ptr(rho1), _ptr(jf), _ptr(out), _ptr(res) if res is not None else None,
+        _stream(stream)))
 
 
 def vpic_migrate_particles(ctx: Context, q: float, m: float, p, np_: int, max_np: int, movers,

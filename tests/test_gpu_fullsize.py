@@ -124,3 +124,19 @@ def test_fullsize_sort_properties(state, order):
         gt |= eq & (c[1:] > c[:-1])
         eq &= c[1:] == c[:-1]
     assert bool(gt.all())
+
+
+def test_fullsize_rho_total_charge(state):
+    """vpic_accumulate_rho on the advanced configs[1] species (the bench's
+    launch configuration; f4 diagnostic): total node charge = q sum w (closed
+    form, conserved by the periodic step) and the mean node charge = one
+    cell's worth."""
+    V, hp, g = state["vpic"], state["hp"], state["g"]
+    for k, sp in enumerate(state["wl"].species):
+        s = hp.species[k]
+        rho = torch.zeros(g.nv, dtype=torch.float32, device="cuda")
+        V.vpic_accumulate_rho(hp.ctx, sp.q, s.p, s.np, rho)
+        tot = float(np.float32(sp.q)) * state["parts"][k]["w"].astype(np.float64).sum()
+        assert abs(rho.double().sum().item() - tot) < 1e-5 * abs(tot)
+        node = rho[torch.from_numpy(g.interior_voxels()).cuda()].double()
+        assert abs(node.mean().item() - tot / g.ncells) < 1e-5 * abs(tot / g.ncells)

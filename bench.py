@@ -51,6 +51,8 @@ def parse():
     ap.add_argument("--kernel", default="auto", choices=["auto", "direct", "tma"])
     ap.add_argument("--field-solve", action="store_true",
                     help="full PIC step: + advance_b/advance_e (self-consistent fields)")
+    ap.add_argument("--concurrent-species", action="store_true",
+                    help="push the species concurrently on two streams (1 CTA/SM each)")
     ap.add_argument("--loopback", action="store_true",
                     help="1 GPU: periodic faces through the NCCL exchange (self peer)")
     ap.add_argument("--no-e2e", action="store_true")
@@ -240,7 +242,8 @@ def our_arm(args, rank, world):
     cap = 1.0 if world == 1 else 1.05
     hp = HotPath(wl, parts, fields, order=order, math=math_mode, deposit=dep, rank=rank,
                  nranks=world, uid=uid, capacity_factor=cap, device=local,
-                 field_solve=args.field_solve, loopback_exchange=args.loopback and world == 1)
+                 field_solve=args.field_solve, loopback_exchange=args.loopback and world == 1,
+                 concurrent_species=args.concurrent_species)
     hp.ctx.set_option(vpic.VPIC_OPT_ADVANCE_KERNEL, {"auto": 0, "direct": 1, "tma": 2}[args.kernel])
     n_local = hp.n_particles
 
@@ -279,6 +282,9 @@ def our_arm(args, rank, world):
     nsp = len(hp.species)
     by_step = [round(sum(adv[(c * S + k) * nsp + j][0] for c in range(args.steps) for j in range(nsp))
                      / (args.steps * nsp), 3) for k in range(S)]
+    by_species = {sp.name: [round(sum(adv[(c * S + k) * nsp + j][0] for c in range(args.steps))
+                                  / args.steps, 3) for k in range(S)]
+                  for j, sp in enumerate(hp.species)}
     adv_np = sum(n for _, n in adv) / len(adv)
     t = torch.tensor([ms, float(pushes_local), float(n_local)], dtype=torch.float64, device=dev)
     if world > 1:
@@ -346,7 +352,8 @@ def our_arm(args, rank, world):
                      "kernel": "k_advance (advance_p, one species per launch)",
                      "alg_bytes_per_launch": alg_bytes, "avg_launch_ms": adv_ms,
                      "share_of_step": adv_share, "frac_of_8TBs": achieved / 8000.0,
-                     "avg_launch_ms_by_step_since_sort": by_step},
+                     "avg_launch_ms_by_step_since_sort": by_step,
+                     "launch_ms_by_species_step": by_species},
         "clocks": clocks,
         "gpu_launches": launches,
         "e2e": e2e,

@@ -86,7 +86,11 @@ enum {
    * particle migration, E/cB halos and the jf plane reduction then run the
    * multi-GPU code path on one GPU, and must reproduce the local periodic
    * wrap.  Validation of the exchange; set once, before any other call. */
-  VPIC_OPT_LOOPBACK_EXCHANGE = 4
+  VPIC_OPT_LOOPBACK_EXCHANGE = 4,
+  /* CTAs per SM of the persistent TMA advance kernel (0 = its default, 2).
+   * 1 lets two advance_p calls (e.g. two species on two streams) be
+   * co-resident, each on half of every SM. */
+  VPIC_OPT_ADVANCE_CTAS_PER_SM = 5
 };
 
 typedef struct {

@@ -113,6 +113,7 @@ int vpic_ctx_create(vpic_ctx **out, const vpic_grid_t *g, int rank, int nranks,
   c->math = MATH_FAST;
   c->deposit = DEP_AUTO;
   c->adv_kernel = ADV_AUTO;
+  c->adv_cps = 0;
   GridK &k = c->gk;
   k.nx = g->nx; k.ny = g->ny; k.nz = g->nz;
   k.sx = g->nx + 2; k.sy = g->ny + 2; k.sxy = k.sx * k.sy;
@@ -175,6 +176,10 @@ int vpic_ctx_set_option(vpic_ctx *c, int option, int64_t value) {
     case VPIC_OPT_ADVANCE_KERNEL:
       if (value < ADV_AUTO || value > ADV_TMA) return VPIC_ERR_INVALID;
       c->adv_kernel = (int)value;
+      return VPIC_OK;
+    case VPIC_OPT_ADVANCE_CTAS_PER_SM:
+      if (value < 0 || value > 2) return VPIC_ERR_INVALID;
+      c->adv_cps = (int)value;
       return VPIC_OK;
     case VPIC_OPT_LOOPBACK_EXCHANGE: {
       if (value != 1 || c->nranks != 1 || c->ex) return VPIC_ERR_INVALID;

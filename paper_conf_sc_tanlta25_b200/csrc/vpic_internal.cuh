@@ -39,6 +39,7 @@ struct vpic_ctx {
   int64_t l2_bytes;
   int64_t tile_sz;
   int math, deposit, adv_kernel;
+  int adv_cps;             // CTAs per SM of k_advance_tma (0 = default)
   bool periodic_local[3];  // axis wraps locally (both faces local periodic)
   vpic::Exchange *ex;      // null when nranks == 1
   // small device scratch owned by the context

@@ -39,7 +39,7 @@ class HotPath:
                  deposit: int = vpic.DEP_AUTO, tile_sz: int = 0, rank: int = 0, nranks: int = 1,
                  uid: bytes = None, capacity_factor: float = 1.0, max_movers: int = 1 << 20,
                  device: Optional[int] = None, field_solve: bool = False, eps0: float = 1.0,
-                 loopback_exchange: bool = False):
+                 loopback_exchange: bool = False, concurrent_species: bool = False):
         vpic.load()
         self.wl = wl
         self.g = wl.grid
@@ -56,6 +56,13 @@ class HotPath:
             self.ctx.set_option(vpic.VPIC_OPT_LOOPBACK_EXCHANGE, 1)
         self.migrate = (nranks > 1 or loopback_exchange
                         or any(b == inputs.BC_ABSORB for b in self.g.pbc))
+        # species pushed concurrently on their own streams, each persistent
+        # kernel on one CTA slot of every SM (not with migration: its counts
+        # synchronise per species)
+        self.concurrent = concurrent_species and not self.migrate and len(wl.species) > 1
+        if self.concurrent:
+            self.ctx.set_option(vpic.VPIC_OPT_ADVANCE_CTAS_PER_SM, 1)
+            self.sp_streams = [torch.cuda.Stream(device=self.dev) for _ in wl.species]
         nv = self.g.nv
         f32 = dict(dtype=torch.float32, device=self.dev)
         self.fields = torch.from_numpy(np.ascontiguousarray(fields)).to(self.dev)
@@ -100,7 +107,22 @@ class HotPath:
         vpic.vpic_load_interpolator(self.ctx, self.fields, self.interp)
         vpic.vpic_clear_accumulator(self.ctx, self.acc)
         stream = torch.cuda.current_stream()
-        for s in self.species:
+        if self.concurrent:
+            ready = torch.cuda.Event()
+            ready.record(stream)
+            for s, st in zip(self.species, self.sp_streams):
+                st.wait_event(ready)
+                if self.record_advance:
+                    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    e0.record(st)
+                vpic.vpic_advance_p(self.ctx, s.q, s.m, s.p, s.np, self.interp, self.acc, s.movers,
+                                    s.movers.shape[0], s.n_movers, s.flags, stream=st)
+                if self.record_advance:
+                    e1.record(st)
+                    self.adv_events.append((e0, e1, s.np))
+            for st in self.sp_streams:
+                stream.wait_stream(st)
+        for s in (() if self.concurrent else self.species):
             if self.record_advance:
                 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 e0.record(stream)

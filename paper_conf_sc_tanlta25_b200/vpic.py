@@ -23,6 +23,7 @@ VPIC_ERR_CUDA, VPIC_ERR_NCCL, VPIC_ERR_UNSUPPORTED = -3, -4, -5
 VPIC_SORT_STANDARD, VPIC_SORT_STRIDED, VPIC_SORT_TILED_STRIDED, VPIC_SORT_NONE = 0, 1, 2, 3
 VPIC_OPT_MATH, VPIC_OPT_DEPOSIT, VPIC_OPT_TILE_SZ, VPIC_OPT_ADVANCE_KERNEL = 0, 1, 2, 3
 VPIC_OPT_LOOPBACK_EXCHANGE = 4
+VPIC_OPT_ADVANCE_CTAS_PER_SM = 5
 MATH_FAST, MATH_IEEE = 0, 1
 DEP_AUTO, DEP_LANE, DEP_WARP = 0, 1, 2
 

@@ -260,6 +260,7 @@ def our_arm(args, rank, world):
     # ---- timed region (device-resident inputs; 17 GB of particles >> 126 MB L2)
     stream = torch.cuda.current_stream()
     hp.adv_events = []
+    hp.sort_events = []
     hp.record_advance = True
     launches0 = vpic.vpic_kernel_launches()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -285,6 +286,10 @@ def our_arm(args, rank, world):
     by_species = {sp.name: [round(sum(adv[(c * S + k) * nsp + j][0] for c in range(args.steps))
                                   / args.steps, 3) for k in range(S)]
                   for j, sp in enumerate(hp.species)}
+    sort_ms = {}
+    for a, b, name in hp.sort_events:
+        sort_ms.setdefault(name, []).append(a.elapsed_time(b))
+    sort_ms = {k: round(sum(v) / len(v), 3) for k, v in sort_ms.items()}
     adv_np = sum(n for _, n in adv) / len(adv)
     t = torch.tensor([ms, float(pushes_local), float(n_local)], dtype=torch.float64, device=dev)
     if world > 1:
@@ -354,6 +359,7 @@ def our_arm(args, rank, world):
                      "share_of_step": adv_share, "frac_of_8TBs": achieved / 8000.0,
                      "avg_launch_ms_by_step_since_sort": by_step,
                      "launch_ms_by_species_step": by_species},
+        "sort_ms_by_species": sort_ms,
         "clocks": clocks,
         "gpu_launches": launches,
         "e2e": e2e,

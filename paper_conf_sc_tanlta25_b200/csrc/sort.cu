@@ -5,8 +5,11 @@
 // B200 design: the paper adjusts keys in O(N) and then calls
 // a generic sort_by_key.  Here every order is produced by stable LSD
 // counting passes with no comparison sort and no nondeterministic atomics:
-//   standard      = stable radix sort of (voxel, index) pairs, 2 passes of
-//                   <= 13-bit digits (chained-scan / decoupled look-back);
+//   standard      = stable radix sort of (voxel, index) pairs, passes of
+//                   <= 8-bit digits (one sweep each: decoupled look-back, the
+//                   tile staged in shared memory in digit order so that every
+//                   digit run is written coalesced), then one gather of the
+//                   32-B records;
 //   strided       = standard, then one stable counting pass by the rank
 //                   r = pos - offset[voxel]        (lexicographic (r, k));
 //   tiled strided = standard, then one stable counting pass by
@@ -22,9 +25,15 @@
 namespace vpic {
 namespace {
 
+#ifndef VPIC_SORT_IPT
+#define VPIC_SORT_IPT 16
+#endif
+#ifndef VPIC_SORT_MINB
+#define VPIC_SORT_MINB 3
+#endif
 constexpr int NT = 256;             // threads per radix CTA
 constexpr int NW = NT / 32;         // warps
-constexpr int IPT = 16;             // items per thread
+constexpr int IPT = VPIC_SORT_IPT;  // items per thread
 constexpr int TILE = NT * IPT;      // 4096 elements per tile
 constexpr int MAX_BITS = 8;         // digit width: 256 buckets, one look-back chain per thread
 constexpr int MAX_PASSES = 4;       // keys up to 32 bits
@@ -207,7 +216,7 @@ __global__ void k_scan_hist(const uint32_t *__restrict__ ghist, uint32_t *__rest
 // publishes its per-digit count and resolves its global offset by decoupled
 // look-back over earlier tiles' status words (flag | count in one u64).
 template <int BITS>
-__global__ void __launch_bounds__(NT, 3)
+__global__ void __launch_bounds__(NT, VPIC_SORT_MINB)
 k_radix_pass(const uint32_t *__restrict__ kin, const uint32_t *__restrict__ vin,
              uint32_t *__restrict__ kout, uint32_t *__restrict__ vout, int64_t n, int shift,
              const uint32_t *__restrict__ dig_off, unsigned long long *__restrict__ status,
@@ -216,6 +225,9 @@ k_radix_pass(const uint32_t *__restrict__ kin, const uint32_t *__restrict__ vin,
   extern __shared__ __align__(16) unsigned char smem[];
   uint16_t *whist = reinterpret_cast<uint16_t *>(smem);                       // [NW][NB]
   uint32_t *tpref = reinterpret_cast<uint32_t *>(smem + NW * NB * 2);          // [NB]
+  uint32_t *tstart = tpref + NB;                                               // [NB]
+  uint32_t *skey = tstart + NB;                                                // [TILE]
+  uint32_t *sval = skey + TILE;                                                // [TILE]
   __shared__ unsigned int s_tile;
   if (threadIdx.x == 0) s_tile = atomicAdd(tile_ctr, 1u);
   for (int i = threadIdx.x; i < NW * NB / 2; i += NT) reinterpret_cast<uint32_t *>(whist)[i] = 0;
@@ -259,6 +271,7 @@ k_radix_pass(const uint32_t *__restrict__ kin, const uint32_t *__restrict__ vin,
       whist[ww * NB + b] = (uint16_t)run;
       run += c;
     }
+    tstart[b] = run;   // tile count of digit b (scanned below)
     unsigned long long *st = status + tile * NB + b;
     uint64_t excl = 0;
     if (tile == 0) {
@@ -267,10 +280,10 @@ k_radix_pass(const uint32_t *__restrict__ kin, const uint32_t *__restrict__ vin,
       st_relaxed(st, FLAG_AGG | run);
       int64_t t = tile - 1;
       while (true) {
-        const unsigned long long s = ld_relaxed(status + t * NB + b);
-        const unsigned long long f = s & (3ull << 62);
+        const unsigned long long sv = ld_relaxed(status + t * NB + b);
+        const unsigned long long f = sv & (3ull << 62);
         if (f == 0) continue;
-        excl += s & VAL_MASK;
+        excl += sv & VAL_MASK;
         if (f == FLAG_INC) break;
         --t;
       }
@@ -279,16 +292,46 @@ k_radix_pass(const uint32_t *__restrict__ kin, const uint32_t *__restrict__ vin,
     tpref[b] = dig_off[b] + (uint32_t)excl;
   }
   __syncthreads();
+  // tile-local exclusive digit offsets (block scan of the NB tile counts)
+  {
+    __shared__ uint32_t wsum[NW];
+    const uint32_t c = threadIdx.x < NB ? tstart[threadIdx.x] : 0u;
+    uint32_t incl = c;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(FULL, incl, o);
+      if (lane >= o) incl += y;
+    }
+    if (lane == 31) wsum[w] = incl;
+    __syncthreads();
+    uint32_t pre = 0;
+    for (int ww = 0; ww < w; ++ww) pre += wsum[ww];
+    if (threadIdx.x < NB) tstart[threadIdx.x] = pre + incl - c;
+    __syncthreads();
+  }
+  // stage the tile in digit order in shared memory, then write each digit's
+  // run with consecutive threads on consecutive addresses (coalesced: one
+  // element-granular scatter per 4 B made the first pass L2-request-bound)
 #pragma unroll
   for (int j = 0; j < IPT; ++j) {
     const int64_t i = wbase + j * 32 + lane;
     if (i < n) {
       const uint32_t d = (key[j] >> shift) & (NB - 1);
       const uint32_t r = (j & 1) ? (rank[j >> 1] >> 16) : (rank[j >> 1] & 0xffffu);
-      const uint32_t pos = tpref[d] + whist[w * NB + d] + r;
-      if (kout) kout[pos] = key[j];
-      vout[pos] = val[j];
+      const uint32_t lp = tstart[d] + whist[w * NB + d] + r;
+      skey[lp] = key[j];
+      sval[lp] = val[j];
     }
+  }
+  __syncthreads();
+  const int64_t t0 = tile * TILE;
+  const int nvalid = (int)(n - t0 < TILE ? n - t0 : (int64_t)TILE);
+  for (int e = threadIdx.x; e < nvalid; e += NT) {
+    const uint32_t k = skey[e];
+    const uint32_t d = (k >> shift) & (NB - 1);
+    const uint32_t pos = tpref[d] + (uint32_t)e - tstart[d];
+    if (kout) kout[pos] = k;
+    vout[pos] = sval[e];
   }
 }
 
@@ -362,14 +405,19 @@ k_gather(const vpic_particle_t *__restrict__ pin, vpic_particle_t *__restrict__ 
 #pragma unroll
     for (int j = 0; j < GATHER_ILP; ++j) {
       const int64_t t = base + lane + 32 * j;
-      sidx[j] = t < nh ? __ldg(perm + (t >> 1)) : 0u;
+      sidx[j] = t < nh ? __ldcs(perm + (t >> 1)) : 0u;
     }
 #pragma unroll
     for (int j = 0; j < GATHER_ILP; ++j) {
       const int64_t t = base + lane + 32 * j;
       // default (evict-normal) caching on purpose: a source line fetched for
       // one record is re-used by the neighbouring output voxels shortly after
-      // (streaming hints made the L2 miss every time: 3.8x read amplification)
+      // (streaming hints made the L2 miss every time).  20 steps after a sort
+      // the electrons of one output voxel come from ~5 z-planes of input
+      // (~350 MB > L2), so DRAM still reads ~3.6x the records; measured
+      // alternatives -- evict_last on these loads, or scattering by the
+      // inverse permutation (whose inversion costs more than it saves) --
+      // were not faster.
       if (t < nh) v[j] = __ldg(src + 2 * (int64_t)sidx[j] + (t & 1));
     }
 #pragma unroll
@@ -460,13 +508,13 @@ template <int BITS>
 cudaError_t radix_pass_bits(const uint32_t *kin, const uint32_t *vin, uint32_t *kout,
                             uint32_t *vout, int64_t n, int shift, const uint32_t *dig_off,
                             unsigned long long *status, unsigned int *ctr, cudaStream_t s) {
-  const size_t smem = (size_t)NW * (1 << BITS) * 2 + (size_t)(1 << BITS) * 4;
+  const size_t smem = (size_t)NW * (1 << BITS) * 2 + (size_t)(1 << BITS) * 8 + (size_t)TILE * 8;
+  const int64_t tiles = (n + TILE - 1) / TILE;
   static bool configured = false;
-  if (!configured) {
+  if (!configured) {   // > 48 KB only for large tiles; set once per instantiation
     cudaFuncSetAttribute(k_radix_pass<BITS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     configured = true;
   }
-  const int64_t tiles = (n + TILE - 1) / TILE;
   k_radix_pass<BITS><<<(unsigned)tiles, NT, smem, s>>>(kin, vin, kout, vout, n, shift, dig_off,
                                                        status, ctr); note_launch();
   return cudaGetLastError();

@@ -86,6 +86,7 @@ class HotPath:
         ws = vpic.vpic_sort_workspace_bytes(self.ctx, max_np, order)
         self.ws = torch.empty(max(ws, 1), dtype=torch.uint8, device=self.dev)
         self.adv_events = []   # (start, end) CUDA events around advance_p, when recording
+        self.sort_events = []  # (start, end, species) around vpic_sort_particles
         self.record_advance = False
 
     # ------------------------------------------------------------ calls --
@@ -97,8 +98,15 @@ class HotPath:
         order = self.order if order is None else order
         if order == vpic.VPIC_SORT_NONE:
             return
+        stream = torch.cuda.current_stream()
         for s in self.species:
+            if self.record_advance:
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(stream)
             vpic.vpic_sort_particles(self.ctx, s.p, s.scratch, s.np, order, self.tile_sz, self.ws)
+            if self.record_advance:
+                e1.record(stream)
+                self.sort_events.append((e0, e1, s.name))
             s.p, s.scratch = s.scratch, s.p
 
     def step(self, do_sort: bool = False):

@@ -3,7 +3,8 @@
 import csv, io, subprocess, sys
 rep = sys.argv[1]
 N = int(sys.argv[2]) if len(sys.argv) > 2 else 40
-out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"],
+extra = sys.argv[3:]   # e.g. -k regex:k_radix --launch-skip 0 -c 1
+out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"] + extra,
                      capture_output=True, text=True).stdout
 rows = list(csv.reader(io.StringIO(out)))
 hdr_i = next(i for i, r in enumerate(rows) if r and r[0] == "Line No")

@@ -53,6 +53,9 @@ def parse():
                     help="full PIC step: + advance_b/advance_e (self-consistent fields)")
     ap.add_argument("--concurrent-species", action="store_true",
                     help="push the species concurrently on two streams (1 CTA/SM each)")
+    ap.add_argument("--device-exchange", action="store_true",
+                    help="device-initiated particle exchange (NCCL symmetric-memory inboxes; "
+                         "needs --loopback on 1 GPU)")
     ap.add_argument("--loopback", action="store_true",
                     help="1 GPU: periodic faces through the NCCL exchange (self peer)")
     ap.add_argument("--no-e2e", action="store_true")
@@ -243,7 +246,8 @@ def our_arm(args, rank, world):
     hp = HotPath(wl, parts, fields, order=order, math=math_mode, deposit=dep, rank=rank,
                  nranks=world, uid=uid, capacity_factor=cap, device=local,
                  field_solve=args.field_solve, loopback_exchange=args.loopback and world == 1,
-                 concurrent_species=args.concurrent_species)
+                 concurrent_species=args.concurrent_species,
+                 device_exchange=args.device_exchange and (world > 1 or args.loopback))
     hp.ctx.set_option(vpic.VPIC_OPT_ADVANCE_KERNEL, {"auto": 0, "direct": 1, "tma": 2}[args.kernel])
     n_local = hp.n_particles
 
@@ -350,6 +354,8 @@ def our_arm(args, rank, world):
                    "deposit": args.deposit, "kernel": args.kernel,
                    "parallelism": "loopback1" if args.loopback and world == 1 else f"domain{world}",
                    "field_solve": bool(args.field_solve),
+                   "exchange": ("device" if args.device_exchange else "nccl")
+                               if (world > 1 or args.loopback) else "none",
                    "l2": f"no flush: inputs ({32 * n_local / 1e9:.1f} GB of particles per GPU) >> 126 MB L2"},
         "per_gpu": value / world,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",

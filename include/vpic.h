@@ -90,7 +90,19 @@ enum {
   /* CTAs per SM of the persistent TMA advance kernel (0 = its default, 2).
    * 1 lets two advance_p calls (e.g. two species on two streams) be
    * co-resident, each on half of every SM. */
-  VPIC_OPT_ADVANCE_CTAS_PER_SM = 5
+  VPIC_OPT_ADVANCE_CTAS_PER_SM = 5,
+  /* Device-initiated particle exchange ("GPU-aware MPI
+   * will reduce the communication overhead"): value >= 1 enables it
+   * with value records per (round, face) inbox (1 = default 2^19).  Needs an
+   * exchange (nranks > 1 or VPIC_OPT_LOOPBACK_EXCHANGE) whose neighbours are
+   * load/store reachable (one NVLink node).  COLLECTIVE: every rank sets it,
+   * with the same value, in the same order of calls.  Then vpic_advance_p
+   * stores each particle that stops on a REMOTE face straight into the
+   * neighbour's inbox (NCCL symmetric memory, NVLink stores), and
+   * vpic_migrate_particles completes the rounds with device-side barriers and
+   * counts: one host synchronisation per call instead of one per round.
+   * Inbox overflow is reported as VPIC_ERR_CAPACITY. */
+  VPIC_OPT_DEVICE_EXCHANGE = 6
 };
 
 typedef struct {

@@ -181,6 +181,11 @@ int vpic_ctx_set_option(vpic_ctx *c, int option, int64_t value) {
       if (value < 0 || value > 2) return VPIC_ERR_INVALID;
       c->adv_cps = (int)value;
       return VPIC_OK;
+    case VPIC_OPT_DEVICE_EXCHANGE: {
+      if (value < 1 || !c->ex) return VPIC_ERR_INVALID;
+      DeviceGuard dg(c->device);
+      return device_exchange_enable(c, value == 1 ? ((int64_t)1 << 19) : value);
+    }
     case VPIC_OPT_LOOPBACK_EXCHANGE: {
       if (value != 1 || c->nranks != 1 || c->ex) return VPIC_ERR_INVALID;
       DeviceGuard dg(c->device);

@@ -5,6 +5,7 @@
 // shared-plane reduction.  Transport: NCCL send/recv (NVLink / NVSwitch) in
 // grouped calls; one process per GPU.
 #include <nccl.h>
+#include <nccl_device.h>
 
 #include <algorithm>
 #include <vector>
@@ -25,6 +26,19 @@ struct Exchange {
   // plane buffers for halo / jf reduction
   float *plane_send = nullptr, *plane_recv = nullptr;
   size_t plane_bytes = 0;
+  // device-initiated exchange (VPIC_OPT_DEVICE_EXCHANGE): inbox window in
+  // NCCL symmetric memory, the device communicator for the LSA barrier, and
+  // device-count driven arrival / hole bookkeeping (no host sync per round)
+  bool di = false;
+  void *di_buf = nullptr;
+  ncclWindow_t di_win = nullptr;
+  ncclDevComm di_dcomm{};
+  bool di_dcomm_ok = false;
+  int64_t di_cap = 0, di_hcap = 0;
+  int64_t *di_ctr = nullptr;          // [0] np [1] H [2] A [3] next movers [4] nlow [5] nsurv [6] np_new [7] base; [8..13] face offsets
+  int32_t *di_flag = nullptr;         // bit 0 inbox full (senders), 1 holes overflow, 2 particles overflow
+  vpic_mover_t *di_arr = nullptr, *di_next = nullptr;
+  uint32_t *di_scr = nullptr;         // hole scratch: tail_dead | low | surv, di_hcap each
 };
 
 namespace {
@@ -187,6 +201,108 @@ int remove_holes(vpic_ctx *c, vpic_particle_t *p, int64_t np, const uint32_t *ho
   return cudaGetLastError() == cudaSuccess ? VPIC_OK : VPIC_ERR_CUDA;
 }
 
+// ---------------------------------------------------- device-initiated --
+struct Peers6 { int lsa[6]; };
+
+__global__ void k_di_peers(ncclWindow_t w, Peers6 pr, unsigned char **out) {
+  for (int f = 0; f < 6; ++f)
+    out[f] = pr.lsa[f] >= 0 ? static_cast<unsigned char *>(ncclGetLsaPointer(w, 0, pr.lsa[f])) : nullptr;
+}
+
+// All ranks of the node reach this point; everything any rank stored into a
+// peer's inbox before (earlier kernels on its stream) is visible after it.
+__global__ void k_lsa_barrier(ncclDevComm dc) {
+  ncclLsaBarrierSession<ncclCoopCta> bar(ncclCoopCta(), dc, ncclTeamTagLsa(), 0);
+  bar.sync(ncclCoopCta(), cuda::memory_order_acq_rel);
+}
+
+__global__ void k_di_set(int64_t *ctr, int64_t np) { ctr[0] = np; ctr[3] = 0; }
+
+// Holes of this round: H = departures in `mv` (device count *hdev).
+__global__ void k_di_holes_prep(int64_t *ctr, const int64_t *hdev, int64_t hcap, int32_t *flag) {
+  int64_t H = *hdev;
+  if (H > hcap) { atomicOr(flag, 2); H = hcap; }
+  ctr[1] = H;
+  ctr[6] = ctr[0] - H;
+  ctr[0] = ctr[6];
+  ctr[4] = 0;
+  ctr[5] = 0;
+}
+__global__ void k_di_mark_tail(const vpic_mover_t *__restrict__ mv, int64_t *ctr,
+                               uint32_t *__restrict__ tail_dead, uint32_t *__restrict__ low) {
+  const int64_t H = ctr[1], np_new = ctr[6];
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < H;
+       k += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t h = (uint32_t)mv[k].idx;
+    if (h >= np_new) tail_dead[h - np_new] = 1;
+    else low[atomicAdd(reinterpret_cast<unsigned long long *>(ctr + 4), 1ull)] = (uint32_t)h;
+  }
+}
+__global__ void k_di_clear(uint32_t *__restrict__ a, const int64_t *ctr) {
+  const int64_t H = ctr[1];
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < H;
+       k += (int64_t)gridDim.x * blockDim.x)
+    a[k] = 0;
+}
+__global__ void k_di_tail_surv(const uint32_t *__restrict__ tail_dead, int64_t *ctr,
+                               uint32_t *__restrict__ surv) {
+  const int64_t H = ctr[1], np_new = ctr[6];
+  for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < H;
+       j += (int64_t)gridDim.x * blockDim.x)
+    if (!tail_dead[j])
+      surv[atomicAdd(reinterpret_cast<unsigned long long *>(ctr + 5), 1ull)] = (uint32_t)(np_new + j);
+}
+__global__ void k_di_backfill(vpic_particle_t *__restrict__ p, const uint32_t *__restrict__ low,
+                              const uint32_t *__restrict__ surv, const int64_t *ctr) {
+  const int64_t n = ctr[4];
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n;
+       k += (int64_t)gridDim.x * blockDim.x)
+    p[low[k]] = p[surv[k]];
+}
+
+// Arrivals of round r: per-face counts -> offsets, append position, reset.
+__global__ void k_di_take(unsigned char *inbox, int r, int64_t cap, int64_t max_np, int64_t *ctr,
+                          int32_t *flag) {
+  if (threadIdx.x != 0) return;
+  int64_t off = 0;
+  for (int f = 0; f < 6; ++f) {
+    unsigned long long *cf = reinterpret_cast<unsigned long long *>(inbox + di_cnt_off(r, f));
+    int64_t a = (int64_t)*cf;
+    if (a > cap) a = cap;     // the senders flagged the overflow
+    ctr[8 + f] = off;
+    off += a;
+    *cf = 0;
+  }
+  const int64_t base = ctr[0];
+  if (base + off > max_np) {  // no room: drop the round's arrivals, report capacity
+    atomicOr(flag, 4);
+    off = 0;
+    for (int f = 0; f < 6; ++f) ctr[8 + f] = 0;
+  }
+  ctr[14] = off;              // (per-face ends for the unpack: offsets + counts)
+  ctr[2] = off;
+  ctr[7] = base;
+  ctr[0] = base + off;
+}
+__global__ void k_di_unpack(const unsigned char *inbox, int r, int64_t cap, const int64_t *ctr,
+                            vpic_particle_t *__restrict__ p, vpic_mover_t *__restrict__ mv) {
+  const int64_t A = ctr[2], base = ctr[7];
+  for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < A;
+       t += (int64_t)gridDim.x * blockDim.x) {
+    int f = 0;
+    while (f < 5 && t >= ctr[8 + f + 1]) ++f;
+    const int64_t k = t - ctr[8 + f];
+    const float4 *rec = reinterpret_cast<const float4 *>(inbox + di_rec_off(r, f, cap, k));
+    const float4 a = rec[0], b = rec[1], d = rec[2];
+    float4 *dst = reinterpret_cast<float4 *>(p + base + t);
+    dst[0] = a;
+    dst[1] = b;
+    vpic_mover_t m;
+    m.dispx = d.x; m.dispy = d.y; m.dispz = d.z; m.idx = (int32_t)(base + t);
+    mv[t] = m;
+  }
+}
+
 }  // namespace
 
 int exchange_create(vpic_ctx *c, const uint8_t *uid) {
@@ -210,6 +326,9 @@ int exchange_create(vpic_ctx *c, const uint8_t *uid) {
 void exchange_destroy(vpic_ctx *c) {
   Exchange *ex = c->ex;
   if (!ex) return;
+  if (ex->di_dcomm_ok) ncclDevCommDestroy(ex->comm, &ex->di_dcomm);
+  if (ex->di_win) ncclCommWindowDeregister(ex->comm, ex->di_win);
+  if (ex->di_buf) ncclMemFree(ex->di_buf);
   if (ex->comm) ncclCommDestroy(ex->comm);
   cudaFree(ex->send);
   cudaFree(ex->recv);
@@ -218,8 +337,122 @@ void exchange_destroy(vpic_ctx *c) {
   cudaFree(ex->plane_recv);
   cudaFree(ex->mv_arr);
   cudaFree(ex->mv_next);
+  cudaFree(ex->di_ctr);
+  cudaFree(ex->di_arr);
+  cudaFree(ex->di_next);
+  cudaFree(ex->di_scr);
   delete ex;
   c->ex = nullptr;
+}
+
+// Collective over the communicator (every rank, same cap): allocate the
+// inbox window in NCCL symmetric memory, register it, create the device
+// communicator (one LSA barrier) and publish the neighbours' inbox addresses
+// to the kernels through GridK.
+int device_exchange_enable(vpic_ctx *c, int64_t cap) {
+  Exchange *ex = c->ex;
+  if (!ex || ex->di || cap <= 0) return VPIC_ERR_INVALID;
+  const size_t bytes = (size_t)di_rec_off(DI_ROUNDS, 0, cap, 0);
+  CKN(ncclMemAlloc(&ex->di_buf, bytes));
+  CKC(cudaMemset(ex->di_buf, 0, DI_HDR));
+  CKN(ncclCommWindowRegister(ex->comm, ex->di_buf, bytes, &ex->di_win, NCCL_WIN_COLL_SYMMETRIC));
+  ncclDevCommRequirements req{};
+  req.lsaBarrierCount = 1;
+  CKN(ncclDevCommCreate(ex->comm, &req, &ex->di_dcomm));
+  ex->di_dcomm_ok = true;
+  Peers6 pr;
+  const ncclTeam_t world = ncclTeamWorld(ex->comm);
+  for (int f = 0; f < 6; ++f) {
+    pr.lsa[f] = -1;
+    if (c->gk.face_kind[f] != FACE_REMOTE) continue;
+    pr.lsa[f] = ncclTeamRankToLsa(ex->comm, world, c->g.nbr_rank[f]);
+    if (pr.lsa[f] < 0) return VPIC_ERR_UNSUPPORTED;   // neighbour not load/store reachable
+  }
+  unsigned char **d_peers = nullptr;
+  CKC(cudaMalloc(&d_peers, 6 * sizeof(void *)));
+  k_di_peers<<<1, 1>>>(ex->di_win, pr, d_peers); note_launch();
+  unsigned char *h_peers[6];
+  const cudaError_t e = cudaMemcpy(h_peers, d_peers, sizeof(h_peers), cudaMemcpyDeviceToHost);
+  cudaFree(d_peers);
+  CKC(e);
+  ex->di_cap = cap;
+  ex->di_hcap = std::max<int64_t>(8 * cap, 1 << 16);
+  CKC(cudaMalloc(&ex->di_ctr, 16 * sizeof(int64_t)));
+  CKC(cudaMemset(ex->di_ctr, 0, 16 * sizeof(int64_t)));
+  CKC(cudaMalloc(&ex->di_flag, sizeof(int32_t)));
+  CKC(cudaMemset(ex->di_flag, 0, sizeof(int32_t)));
+  CKC(cudaMalloc(&ex->di_arr, (size_t)6 * cap * sizeof(vpic_mover_t)));
+  CKC(cudaMalloc(&ex->di_next, (size_t)6 * cap * sizeof(vpic_mover_t)));
+  CKC(cudaMalloc(&ex->di_scr, (size_t)3 * ex->di_hcap * sizeof(uint32_t)));
+  for (int f = 0; f < 6; ++f) c->gk.di_peer[f] = h_peers[f];
+  c->gk.di_cap = cap;
+  c->gk.di_flag = ex->di_flag;
+  c->gk.di_round = 0;
+  c->gk.di_on = 1;
+  ex->di = true;
+  return VPIC_OK;
+}
+
+namespace {
+
+// Remove this round's departures (device count) by back-filling from the tail.
+int di_remove_holes(vpic_ctx *c, vpic_particle_t *p, const vpic_mover_t *mv, const int64_t *hdev,
+                    cudaStream_t s) {
+  Exchange *ex = c->ex;
+  const unsigned B = (unsigned)c->num_sms * 4;
+  uint32_t *tail_dead = ex->di_scr, *low = ex->di_scr + ex->di_hcap, *surv = ex->di_scr + 2 * ex->di_hcap;
+  k_di_holes_prep<<<1, 1, 0, s>>>(ex->di_ctr, hdev, ex->di_hcap, ex->di_flag); note_launch();
+  k_di_clear<<<B, 256, 0, s>>>(tail_dead, ex->di_ctr); note_launch();
+  k_di_mark_tail<<<B, 256, 0, s>>>(mv, ex->di_ctr, tail_dead, low); note_launch();
+  k_di_tail_surv<<<B, 256, 0, s>>>(tail_dead, ex->di_ctr, surv); note_launch();
+  k_di_backfill<<<B, 256, 0, s>>>(p, low, surv, ex->di_ctr); note_launch();
+  return cudaGetLastError() == cudaSuccess ? VPIC_OK : VPIC_ERR_CUDA;
+}
+
+}  // namespace
+
+// Device-initiated migration (f4).  The movers' particles were already
+// stored into the neighbours' round-0 inboxes by advance_p (REMOTE faces) or
+// are absorbed; every round: remove this rank's departures, LSA barrier (all
+// round-r stores landed), append the arrivals, continue their move -- whose
+// departures k_move_movers stores into the round r+1 inboxes.  Counts stay
+// on the device; one host synchronisation at the end (the new np).
+int migrate_di(vpic_ctx *c, float qsp, vpic_particle_t *p, int64_t *np_io, int64_t max_np,
+               vpic_mover_t *movers, const int64_t *n_movers, float *acc, cudaStream_t s) {
+  Exchange *ex = c->ex;
+  int32_t *d_flags = reinterpret_cast<int32_t *>(c->d_count + 1);
+  CKC(cudaMemsetAsync(d_flags, 0, 4, s));
+  k_di_set<<<1, 1, 0, s>>>(ex->di_ctr, *np_io); note_launch();
+  if (int rc = di_remove_holes(c, p, movers, n_movers, s)) return rc;
+  const int64_t acap = 6 * ex->di_cap;
+  const unsigned B = (unsigned)c->num_sms * 4;
+  unsigned char *inbox = static_cast<unsigned char *>(ex->di_buf);
+  for (int r = 0; r < DI_ROUNDS; ++r) {
+    k_lsa_barrier<<<1, 128, 0, s>>>(ex->di_dcomm); note_launch();
+    k_di_take<<<1, 32, 0, s>>>(inbox, r, ex->di_cap, max_np, ex->di_ctr, ex->di_flag); note_launch();
+    k_di_unpack<<<B, 256, 0, s>>>(inbox, r, ex->di_cap, ex->di_ctr, p, ex->di_arr); note_launch();
+    CKC(cudaMemsetAsync(ex->di_ctr + 3, 0, 8, s));
+    // departures of the arrivals go to the round r+1 inboxes (dropped after the last round)
+    cudaError_t e = (c->math == MATH_IEEE)
+        ? launch_move_movers_ieee(c, qsp, p, ex->di_arr, acap, acc, ex->di_next, acap, ex->di_ctr + 3,
+                                  d_flags, s, ex->di_ctr + 2, r + 1)
+        : launch_move_movers_fast(c, qsp, p, ex->di_arr, acap, acc, ex->di_next, acap, ex->di_ctr + 3,
+                                  d_flags, s, ex->di_ctr + 2, r + 1);
+    CKC(e);
+    if (int rc = di_remove_holes(c, p, ex->di_next, ex->di_ctr + 3, s)) return rc;
+  }
+  int64_t h_np = 0;
+  int32_t h_fl[2] = {0, 0};
+  CKC(cudaMemcpyAsync(&h_np, ex->di_ctr, 8, cudaMemcpyDeviceToHost, s));
+  CKC(cudaMemcpyAsync(&h_fl[0], d_flags, 4, cudaMemcpyDeviceToHost, s));
+  CKC(cudaMemcpyAsync(&h_fl[1], ex->di_flag, 4, cudaMemcpyDeviceToHost, s));
+  CKC(cudaStreamSynchronize(s));
+  *np_io = h_np;
+  if (h_fl[0] || h_fl[1]) {
+    CKC(cudaMemsetAsync(ex->di_flag, 0, 4, s));
+    return VPIC_ERR_CAPACITY;
+  }
+  return VPIC_OK;
 }
 
 // Up to 3 rounds: pack movers per face, exchange counts, exchange records,
@@ -229,6 +462,7 @@ void exchange_destroy(vpic_ctx *c) {
 int migrate(vpic_ctx *c, float qsp, float msp, vpic_particle_t *p, int64_t *np_io, int64_t max_np,
             vpic_mover_t *movers, const int64_t *n_movers, float *acc, cudaStream_t s) {
   (void)msp;
+  if (c->ex && c->ex->di) return migrate_di(c, qsp, p, np_io, max_np, movers, n_movers, acc, s);
   int64_t M = 0;
   CKC(cudaMemcpyAsync(&M, n_movers, 8, cudaMemcpyDeviceToHost, s));
   CKC(cudaStreamSynchronize(s));

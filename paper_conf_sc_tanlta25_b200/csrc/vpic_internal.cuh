@@ -19,7 +19,25 @@ struct GridK {
   float dt, cvac;
   // per face: 0 = local neighbour/wrap, 1 = reflect, 2 = absorb, 3 = remote
   int32_t face_kind[6];
+  // device-initiated exchange (VPIC_OPT_DEVICE_EXCHANGE):
+  // a particle stopping on a REMOTE face f is stored straight into the
+  // inbox window of nbr_rank[f] (NCCL symmetric memory, LSA address di_peer[f])
+  unsigned char *di_peer[6];
+  int64_t di_cap;            // records per (round, face) inbox
+  int32_t *di_flag;          // local: bit 0 set when an inbox was full
+  int32_t di_round;          // migration round of this launch's departures
+  int32_t di_on;
 };
+
+// inbox window layout: counters [DI_ROUNDS][6] (u64), then records
+// [DI_ROUNDS][6][di_cap] x 48 B (position record, momentum record, remaining
+// displacement); the round-r counter of face f counts arrivals through MY face f
+constexpr int DI_ROUNDS = 3;
+constexpr int64_t DI_HDR = 256;
+__host__ __device__ inline int64_t di_cnt_off(int r, int f) { return 8 * (int64_t)(r * 6 + f); }
+__host__ __device__ inline int64_t di_rec_off(int r, int f, int64_t cap, int64_t k) {
+  return DI_HDR + 48 * ((int64_t)(r * 6 + f) * cap + k);
+}
 
 enum FaceKind { FACE_LOCAL = 0, FACE_REFLECT = 1, FACE_ABSORB = 2, FACE_REMOTE = 3 };
 
@@ -68,14 +86,18 @@ cudaError_t launch_advance_p_ieee(const vpic_ctx *c, float qsp, float msp, vpic_
                                   vpic_mover_t *movers, int64_t max_movers, int64_t *n_movers,
                                   int32_t *flags, cudaStream_t s);
 // move_p of a list of movers (incoming particles after migration)
+// n_in_dev (nullable): device count, n_in then only bounds it; di_round: the
+// migration round of the departures (device-initiated exchange only)
 cudaError_t launch_move_movers_fast(const vpic_ctx *c, float qsp, vpic_particle_t *p,
                                     const vpic_mover_t *in, int64_t n_in, float *acc,
                                     vpic_mover_t *out, int64_t max_out, int64_t *n_out,
-                                    int32_t *flags, cudaStream_t s);
+                                    int32_t *flags, cudaStream_t s,
+                                    const int64_t *n_in_dev = nullptr, int di_round = 0);
 cudaError_t launch_move_movers_ieee(const vpic_ctx *c, float qsp, vpic_particle_t *p,
                                     const vpic_mover_t *in, int64_t n_in, float *acc,
                                     vpic_mover_t *out, int64_t max_out, int64_t *n_out,
-                                    int32_t *flags, cudaStream_t s);
+                                    int32_t *flags, cudaStream_t s,
+                                    const int64_t *n_in_dev = nullptr, int di_round = 0);
 
 cudaError_t launch_fill_ghosts(const vpic_ctx *c, float *fields, cudaStream_t s);
 cudaError_t launch_load_interp(const vpic_ctx *c, const float *fields, float *interp,
@@ -107,6 +129,7 @@ void exchange_destroy(vpic_ctx *c);
 // dir = +1: fill the +x/+y/+z ghost planes from the +neighbours' plane 1;
 // dir = -1: fill the -x/-y/-z ghost planes from the -neighbours' plane n.
 int halo_fields(vpic_ctx *c, float *fields, cudaStream_t s, int dir = +1);
+int device_exchange_enable(vpic_ctx *c, int64_t cap);
 int reduce_jf(vpic_ctx *c, float *jf, cudaStream_t s);
 
 }  // namespace vpic

@@ -88,13 +88,17 @@ def _multiset(a):
     return np.sort(np.ascontiguousarray(a).view(np.dtype((np.void, 32))).ravel())
 
 
+@pytest.mark.parametrize("device_exchange", [False, True], ids=["nccl", "device"])
 @pytest.mark.parametrize("field_solve,steps", [(False, 3), (True, 1)])
-def test_loopback_exchange_matches_periodic(V, field_solve, steps):
+def test_loopback_exchange_matches_periodic(V, field_solve, steps, device_exchange):
     """VPIC_OPT_LOOPBACK_EXCHANGE sends every periodic crossing, E/cB halo and
     jf shared plane through the NCCL exchange (one-rank communicator, self
     peer): the multi-GPU code path on one GPU.  It must reproduce the local
     periodic wrap: particles bit-exact as multisets (migration reorders
-    them), jf and fields within the atomic-reordering tolerance."""
+    them), jf and fields within the atomic-reordering tolerance.  "device":
+    the device-initiated exchange (f4) -- the push stores movers into the
+    (self) neighbour's symmetric-memory inbox, rounds synchronised on the
+    device."""
     from paper_conf_sc_tanlta25_b200.pic import HotPath
     g = inputs.GridSpec(8, 6, 5, dt=0.5)
     wl = inputs.Workload("loopback", g, [inputs.Species("electron", -1.0, 1.0, 0.6),
@@ -104,7 +108,8 @@ def test_loopback_exchange_matches_periodic(V, field_solve, steps):
     runs = []
     for loop in (False, True):
         hp = HotPath(wl, parts, fields, math=V.MATH_IEEE, field_solve=field_solve,
-                     loopback_exchange=loop, capacity_factor=1.0)
+                     loopback_exchange=loop, capacity_factor=1.0,
+                     device_exchange=loop and device_exchange, inbox_cap=4096)
         for _ in range(steps):
             hp.step()
         torch.cuda.synchronize()
@@ -123,3 +128,17 @@ def test_loopback_exchange_matches_periodic(V, field_solve, steps):
     assert np.abs(fa - fb).max() <= 1e-5 * max(1.0, np.abs(fa).max())
     if not field_solve:
         assert np.array_equal(fa, fb)       # static fields: halos move bytes only
+
+
+def test_device_exchange_inbox_overflow_reported(V):
+    """An inbox smaller than one round's arrivals: the push keeps going,
+    vpic_migrate_particles reports VPIC_ERR_CAPACITY (no silent loss)."""
+    from paper_conf_sc_tanlta25_b200.pic import HotPath
+    g = inputs.GridSpec(6, 5, 4, dt=0.5)
+    wl = inputs.Workload("overflow", g, [inputs.Species("electron", -1.0, 1.0, 0.8)], 60, 1, 0)
+    parts = inputs.make_species_particles(wl)
+    hp = HotPath(wl, parts, inputs.make_fields(g, 0.05), loopback_exchange=True,
+                 device_exchange=True, inbox_cap=2, capacity_factor=1.0)
+    with pytest.raises(V.VpicError) as ei:
+        hp.step()
+    assert ei.value.status == -2      # VPIC_ERR_CAPACITY

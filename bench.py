@@ -53,9 +53,9 @@ def parse():
                     help="full PIC step: + advance_b/advance_e (self-consistent fields)")
     ap.add_argument("--concurrent-species", action="store_true",
                     help="push the species concurrently on two streams (1 CTA/SM each)")
-    ap.add_argument("--device-exchange", action="store_true",
-                    help="device-initiated particle exchange (NCCL symmetric-memory inboxes; "
-                         "needs --loopback on 1 GPU)")
+    ap.add_argument("--exchange", default="auto", choices=["auto", "nccl", "device"],
+                    help="particle exchange when there is one (N>1 or --loopback): device-initiated "
+                         "(symmetric-memory inboxes, the default) or NCCL send/recv rounds")
     ap.add_argument("--loopback", action="store_true",
                     help="1 GPU: periodic faces through the NCCL exchange (self peer)")
     ap.add_argument("--no-e2e", action="store_true")
@@ -247,7 +247,7 @@ def our_arm(args, rank, world):
                  nranks=world, uid=uid, capacity_factor=cap, device=local,
                  field_solve=args.field_solve, loopback_exchange=args.loopback and world == 1,
                  concurrent_species=args.concurrent_species,
-                 device_exchange=args.device_exchange and (world > 1 or args.loopback))
+                 device_exchange=args.exchange in ("auto", "device") and (world > 1 or args.loopback))
     hp.ctx.set_option(vpic.VPIC_OPT_ADVANCE_KERNEL, {"auto": 0, "direct": 1, "tma": 2}[args.kernel])
     n_local = hp.n_particles
 
@@ -354,7 +354,7 @@ def our_arm(args, rank, world):
                    "deposit": args.deposit, "kernel": args.kernel,
                    "parallelism": "loopback1" if args.loopback and world == 1 else f"domain{world}",
                    "field_solve": bool(args.field_solve),
-                   "exchange": ("device" if args.device_exchange else "nccl")
+                   "exchange": ("nccl" if args.exchange == "nccl" else "device")
                                if (world > 1 or args.loopback) else "none",
                    "l2": f"no flush: inputs ({32 * n_local / 1e9:.1f} GB of particles per GPU) >> 126 MB L2"},
         "per_gpu": value / world,

@@ -415,9 +415,10 @@ k_gather(const vpic_particle_t *__restrict__ pin, vpic_particle_t *__restrict__ 
       // (streaming hints made the L2 miss every time).  20 steps after a sort
       // the electrons of one output voxel come from ~5 z-planes of input
       // (~350 MB > L2), so DRAM still reads ~3.6x the records; measured
-      // alternatives -- evict_last on these loads, or scattering by the
-      // inverse permutation (whose inversion costs more than it saves) --
-      // were not faster.
+      // alternatives -- evict_last on these loads, scattering by the inverse
+      // permutation (whose inversion costs more than it saves), gathering in
+      // (y-tile, z) segment order so that a segment's sources (~50 MB) stay
+      // in L2 (still 31 GB read, 5% L2 hits) -- were not faster.
       if (t < nh) v[j] = __ldg(src + 2 * (int64_t)sidx[j] + (t & 1));
     }
 #pragma unroll

@@ -306,8 +306,11 @@ def our_arm(args, rank, world):
         ms_max, pushes, ntot = ms, float(pushes_local), float(n_local)
     value = pushes / (ms_max / 1e3)
 
-    # ---- e2e: host (pinned) -> device inputs and device -> host results inside the timed region
-    e2e = None
+    # ---- e2e: host (pinned) -> device inputs and device -> host results inside the timed region.
+    # e2e: every step uploads the particles + fields and reads back the step's
+    # result, jf (the current density the push produces for the field solver);
+    # e2e_state_roundtrip additionally reads every particle back each step.
+    e2e = e2e_rt = None
     if not args.no_e2e and not args.profile:
         host_in = [torch.from_numpy(np.ascontiguousarray(p).view(np.float32).reshape(-1, 8)).pin_memory()
                    for p in parts]
@@ -315,23 +318,29 @@ def our_arm(args, rank, world):
         f_host = torch.from_numpy(fields).pin_memory()
         jf_host = torch.empty(tuple(hp.jf.shape), dtype=torch.float32, pin_memory=True)
         h2d = sum(h.numel() * 4 for h in host_in) + f_host.numel() * 4
-        d2h = sum(h.numel() * 4 for h in host_out) + jf_host.numel() * 4
-        torch.cuda.synchronize()
-        barrier()
-        a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        a0.record(stream)
-        e2e_pushes = hp.run_host_cycles(host_in, host_out, f_host, jf_host, args.steps, S)
-        a1.record(stream)
-        torch.cuda.synchronize()
-        barrier()
-        ems = a0.elapsed_time(a1)
-        et = torch.tensor([ems, float(e2e_pushes)], dtype=torch.float64, device=dev)
-        if world > 1:
-            em = et.clone(); dist.all_reduce(em, op=dist.ReduceOp.MAX)
-            es = et.clone(); dist.all_reduce(es, op=dist.ReduceOp.SUM)
-            ems, e2e_pushes = float(em[0]), float(es[1])
-        e2e = {"value": e2e_pushes / (ems / 1e3), "unit": UNIT, "h2d_bytes_per_step": h2d,
-               "d2h_bytes_per_step": d2h}
+
+        def timed_e2e(outs):
+            torch.cuda.synchronize()
+            barrier()
+            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a0.record(stream)
+            n = hp.run_host_cycles(host_in, outs, f_host, jf_host, args.steps, S)
+            a1.record(stream)
+            torch.cuda.synchronize()
+            barrier()
+            t = torch.tensor([a0.elapsed_time(a1), float(n)], dtype=torch.float64, device=dev)
+            if world > 1:
+                tm = t.clone(); dist.all_reduce(tm, op=dist.ReduceOp.MAX)
+                ts = t.clone(); dist.all_reduce(ts, op=dist.ReduceOp.SUM)
+                t = torch.stack([tm[0], ts[1]])
+            return float(t[1]) / (float(t[0]) / 1e3)
+
+        e2e = {"value": timed_e2e(None), "unit": UNIT, "h2d_bytes_per_step": h2d,
+               "d2h_bytes_per_step": jf_host.numel() * 4,
+               "result": "jf (current density) read back every step"}
+        e2e_rt = {"value": timed_e2e(host_out), "unit": UNIT, "h2d_bytes_per_step": h2d,
+                  "d2h_bytes_per_step": sum(h.numel() * 4 for h in host_out) + jf_host.numel() * 4,
+                  "result": "every particle and jf read back every step"}
 
     if rank != 0:
         return
@@ -369,6 +378,7 @@ def our_arm(args, rank, world):
         "clocks": clocks,
         "gpu_launches": launches,
         "e2e": e2e,
+        "e2e_state_roundtrip": e2e_rt,
     }
     if not args.no_cpu_baseline and not args.profile and world == 1:
         out["cpu_baseline"] = cpu_baseline(args)

@@ -160,8 +160,8 @@ class HotPath:
     # ------------------------------------------------------- host <-> device --
     def run_host_cycles(self, host_in, host_out, fields_host, jf_host, n_cycles: int, S: int):
         """Stream `n_cycles` sort periods from pinned host memory: every cycle
-        uploads its particle and field inputs and downloads its particles and
-        jf.  The H2D of cycle k+1 and the D2H of cycle k run on copy streams
+        uploads its particle and field inputs and downloads jf and, unless
+        host_out is None, its particles.  The H2D of cycle k+1 and the D2H of cycle k run on copy streams
         under the neighbouring cycles' compute; 4 device particle buffers per
         species rotate through input / sort scratch / result / spare.
         Returns the pushes done (particles x PIC steps)."""
@@ -214,7 +214,7 @@ class HotPath:
                    for j in range(nsp)]
             with torch.cuda.stream(d2h):
                 d2h.wait_event(ev_c)
-                for j, sp in enumerate(self.species):
+                for j, sp in enumerate(self.species if host_out is not None else ()):
                     n = min(sp.np, host_out[j].shape[0])
                     host_out[j][:n].copy_(sp.p[:n], non_blocking=True)
                 jf_host.copy_(jstage[k % 2], non_blocking=True)

@@ -38,6 +38,16 @@ def dev_particles(V, p):
     return V.particles_to_device(p)
 
 
+def harris_small():
+    """configs[2]'s Harris sheet (sech^2 density, tanh cB_x, reflecting z,
+    drifting species) on a 24x8x32 grid, 40 ppc mean: ~4x the background
+    density in the sheet -- the contention case."""
+    from dataclasses import replace
+    wl = inputs.config(2)
+    wh = replace(wl, grid=inputs.GridSpec(24, 8, 32, pbc=wl.grid.pbc), ppc=40)
+    return wh, inputs.make_species_particles(wh)
+
+
 # ------------------------------------------------------------------ sort --
 def sort_cases():
     out = []
@@ -53,6 +63,8 @@ def sort_cases():
     out.append(("warp_minus_one", g, inputs.random_particles(g, 31, 6)))
     g2 = inputs.GridSpec(32, 32, 32)
     out.append(("many_tiles", g2, inputs.shuffle(inputs.random_particles(g2, 200000, 7), 8)))
+    wh, ph = harris_small()
+    out.append(("harris_sheet", wh.grid, inputs.shuffle(ph[1], 9)))
     return out
 
 
@@ -119,7 +131,11 @@ def adv_cases():
     gr = inputs.GridSpec(5, 6, 7)
     out.append(("periodic_hot_ragged", gr, inputs.random_particles(gr, 12345, 12, u_scale=1.2), 0.7,
                 1.3, inputs.make_fields(gr, 0.2, seed=4)))
+    wh, ph = harris_small()
+    out.append(("harris_sheet_electrons", wh.grid, ph[0], -1.0, 1.0,
+                inputs.make_fields(wh.grid, 0.01, kind="harris")))
     return out
+
 
 
 def run_both(V, orc, g, p, q, m, fields, math, deposit, kernel=0):

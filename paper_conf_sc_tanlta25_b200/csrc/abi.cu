@@ -124,6 +124,8 @@ int vpic_ctx_create(vpic_ctx **out, const vpic_grid_t *g, int rank, int nranks,
   k.cdt_dz = g->cvac * g->dt / g->dz;
   k.dt = g->dt;
   k.cvac = g->cvac;
+  set_magic((uint32_t)k.sx, k.mag_sx, k.sh_sx);
+  set_magic((uint32_t)k.sxy, k.mag_sxy, k.sh_sxy);
   for (int f = 0; f < 6; ++f) {
     if (g->pbc[f] == VPIC_BC_REFLECT) k.face_kind[f] = FACE_REFLECT;
     else if (g->pbc[f] == VPIC_BC_ABSORB) k.face_kind[f] = FACE_ABSORB;

@@ -19,6 +19,8 @@ struct GridK {
   float dt, cvac;
   // per face: 0 = local neighbour/wrap, 1 = reflect, 2 = absorb, 3 = remote
   int32_t face_kind[6];
+  // v / sx and v / sxy for 0 <= v < 2^31 as umulhi(v, mag) >> sh (set_magic)
+  uint32_t mag_sx, sh_sx, mag_sxy, sh_sxy;
   // device-initiated exchange (VPIC_OPT_DEVICE_EXCHANGE):
   // a particle stopping on a REMOTE face f is stored straight into the
   // inbox window of nbr_rank[f] (NCCL symmetric memory, LSA address di_peer[f])
@@ -28,6 +30,17 @@ struct GridK {
   int32_t di_round;          // migration round of this launch's departures
   int32_t di_on;
 };
+
+// Round-up reciprocal for exact unsigned division of n < 2^31 by d >= 2:
+// s = ceil(log2 d) - 1, m = ceil(2^(32+s) / d) < 2^32; then n / d ==
+// umulhi(n, m) >> s (the error e = m d - 2^(32+s) < d <= 2^(s+1) keeps
+// n e < 2^(32+s)).
+inline void set_magic(uint32_t d, uint32_t &m, uint32_t &s) {
+  uint32_t k = 0;
+  while ((1ull << (k + 1)) < d) ++k;          // 2^k < d <= 2^(k+1)
+  s = k;
+  m = (uint32_t)(((1ull << (32 + k)) + d - 1) / d);
+}
 
 // inbox window layout: counters [DI_ROUNDS][6] (u64), then records
 // [DI_ROUNDS][6][di_cap] x 48 B (position record, momentum record, remaining

@@ -134,6 +134,10 @@ def adv_cases():
     wh, ph = harris_small()
     out.append(("harris_sheet_electrons", wh.grid, ph[0], -1.0, 1.0,
                 inputs.make_fields(wh.grid, 0.01, kind="harris")))
+    # random order on 40^3 voxels: every warp's items in distinct voxels
+    gs = inputs.GridSpec(40, 40, 40)
+    out.append(("scattered_cache_overflow", gs, inputs.random_particles(gs, 150000, 13, u_scale=0.5),
+                -1.0, 1.0, inputs.make_fields(gs, 0.02, seed=5)))
     return out
 
 
@@ -163,7 +167,7 @@ def run_both(V, orc, g, p, q, m, fields, math, deposit, kernel=0):
 
 
 @pytest.mark.parametrize("case", adv_cases(), ids=lambda c: c[0])
-@pytest.mark.parametrize("deposit", [1, 2])
+@pytest.mark.parametrize("deposit", [1, 2], ids=["lane", "warp"])
 @pytest.mark.parametrize("kernel", [1, 2], ids=["direct", "tma"])
 def test_advance_ieee_bitexact(V, orc, case, deposit, kernel):
     name, g, p, q, m, f = case
@@ -177,10 +181,16 @@ def test_advance_ieee_bitexact(V, orc, case, deposit, kernel):
 
 
 @pytest.mark.parametrize("case", adv_cases(), ids=lambda c: c[0])
-@pytest.mark.parametrize("deposit", [1, 2])
+@pytest.mark.parametrize("deposit", [1, 2], ids=["lane", "warp"])
 @pytest.mark.parametrize("kernel", [1, 2], ids=["direct", "tma"])
 def test_advance_fast_tolerance(V, orc, case, deposit, kernel):
     name, g, p, q, m, f = case
+    if name == "scattered_cache_overflow":
+        # ~2 particles per voxel: an entry can hold ONE partial q ux (1 - dy)...
+        # with dy ~ +-1, whose FMA-contracted value differs from the oracle's
+        # by ~ulp(q ux), far above 1e-5 of the cancelled partial (T1 bounds
+        # reordering, not FAST-mode arithmetic); IEEE mode checks this case
+        pytest.skip("IEEE-only case (sparse entries: FAST-mode FMA vs T1)")
     r = run_both(V, orc, g, p, q, m, f, V.MATH_FAST, deposit, kernel)
     assert_particles_close(g, r["p"], r["p_o"], u_of(p), kick_bound(g, p, q, m, r["interp_o"]))
     assert_acc_close(r["acc"], r["acc_o"], r["acc_abs"])

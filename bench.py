@@ -56,6 +56,9 @@ def parse():
     ap.add_argument("--exchange", default="auto", choices=["auto", "nccl", "device"],
                     help="particle exchange when there is one (N>1 or --loopback): device-initiated "
                          "(symmetric-memory inboxes, the default) or NCCL send/recv rounds")
+    ap.add_argument("--migration", default="auto", choices=["auto", "rounds", "single"],
+                    help="with an exchange: single-round 26-neighbour migration (moves finished in "
+                         "the ghost layer; the default) or up to 3 face rounds")
     ap.add_argument("--loopback", action="store_true",
                     help="1 GPU: periodic faces through the NCCL exchange (self peer)")
     ap.add_argument("--no-e2e", action="store_true")
@@ -247,7 +250,8 @@ def our_arm(args, rank, world):
                  nranks=world, uid=uid, capacity_factor=cap, device=local,
                  field_solve=args.field_solve, loopback_exchange=args.loopback and world == 1,
                  concurrent_species=args.concurrent_species,
-                 device_exchange=args.exchange in ("auto", "device") and (world > 1 or args.loopback))
+                 device_exchange=args.exchange in ("auto", "device") and (world > 1 or args.loopback),
+                 single_round=args.migration in ("auto", "single") and (world > 1 or args.loopback))
     hp.ctx.set_option(vpic.VPIC_OPT_ADVANCE_KERNEL, {"auto": 0, "direct": 1, "tma": 2}[args.kernel])
     n_local = hp.n_particles
 
@@ -367,6 +371,8 @@ def our_arm(args, rank, world):
                    "field_solve": bool(args.field_solve),
                    "exchange": ("nccl" if args.exchange == "nccl" else "device")
                                if (world > 1 or args.loopback) else "none",
+                   "migration": ("rounds" if args.migration == "rounds" else "single")
+                                if (world > 1 or args.loopback) else "none",
                    "l2": f"no flush: inputs ({32 * n_local / 1e9:.1f} GB of particles per GPU) >> 126 MB L2"},
         "per_gpu": value / world,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",

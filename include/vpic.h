@@ -102,7 +102,24 @@ enum {
    * vpic_migrate_particles completes the rounds with device-side barriers and
    * counts: one host synchronisation per call instead of one per round.
    * Inbox overflow is reported as VPIC_ERR_CAPACITY. */
-  VPIC_OPT_DEVICE_EXCHANGE = 6
+  VPIC_OPT_DEVICE_EXCHANGE = 6,
+  /* Single-round migration (SURVEY.md §8(e) alternative (2); the paper's
+   * exchange is "non-blocking point-to-point with up to six neighbors",
+   * P:55): value 1.  Needs an exchange; COLLECTIVE (every rank, same order);
+   * set it before VPIC_OPT_DEVICE_EXCHANGE and before any vpic_advance_p.
+   * Then a particle crossing a REMOTE face does not stop there: it finishes
+   * its move in this rank's ghost layer (the move is < 1 cell per axis),
+   * depositing into the ghost voxels of acc, and leaves from the ghost voxel
+   * it ends in -- to one of up to 26 neighbours (faces, edges, corners;
+   * ranks found by composing the face neighbours x, then y, then z).
+   * vpic_migrate_particles then makes ONE exchange (NCCL, or stores into the
+   * neighbours' inboxes from advance_p itself with VPIC_OPT_DEVICE_EXCHANGE),
+   * appends the arrivals (nothing left to move), and adds acc's ghost layer
+   * into the neighbours' boundary voxels (axis by axis, then zeroes it): so
+   * call vpic_migrate_particles after EVERY species' vpic_advance_p, before
+   * vpic_unload_accumulator.  Reproduces the 3-round path's particles and
+   * currents (the latter up to float summation order). */
+  VPIC_OPT_SINGLE_ROUND_MIGRATION = 7
 };
 
 typedef struct {
@@ -189,7 +206,9 @@ int vpic_clear_accumulator(vpic_ctx *ctx, float *acc, void *stream);
  * Particles are updated in place.  A particle that reaches a REMOTE or ABSORB
  * face stops there (offset exactly +-1 on the face, p.i = 8*voxel + face) and
  * appends a mover {remaining displacement, index} at movers[atomic n_movers++];
- * the append order is unspecified.
+ * the append order is unspecified.  (VPIC_OPT_SINGLE_ROUND_MIGRATION: a
+ * particle ending its move in the ghost layer gets p.i = -1 - ghost voxel and
+ * a mover with zero displacement; absorbed ones as above.)
  *   n_movers   device int64, in/out (not reset by this call);
  *   flags      device int32, nullable: bit 0 set if a mover was dropped
  *              because *n_movers reached max_movers. */
@@ -268,7 +287,9 @@ int vpic_continuity_residual(vpic_ctx *ctx, const float *rho0, const float *rho1
  * acc) and are appended; absorbed and departed particles are removed by
  * back-filling from the end.  *np (HOST) is updated.  SYNCHRONISES `stream`
  * (it reads mover counts).  Fails with VPIC_ERR_CAPACITY if the arrivals would
- * exceed max_np. */
+ * exceed max_np.  With VPIC_OPT_SINGLE_ROUND_MIGRATION: one exchange with up
+ * to 26 neighbours, arrivals appended with their move already complete, then
+ * acc's ghost layer added into the neighbours' boundary voxels and zeroed. */
 int vpic_migrate_particles(vpic_ctx *ctx, float q, float m, vpic_particle_t *p, int64_t *np,
                            int64_t max_np, vpic_mover_t *movers, const int64_t *n_movers,
                            float *acc, void *stream);

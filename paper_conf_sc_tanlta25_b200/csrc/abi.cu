@@ -183,6 +183,11 @@ int vpic_ctx_set_option(vpic_ctx *c, int option, int64_t value) {
       if (value < 0 || value > 2) return VPIC_ERR_INVALID;
       c->adv_cps = (int)value;
       return VPIC_OK;
+    case VPIC_OPT_SINGLE_ROUND_MIGRATION: {
+      if (value != 1 || !c->ex || c->gk.ghost_mig) return VPIC_ERR_INVALID;
+      DeviceGuard dg(c->device);
+      return ghost_migration_enable(c);
+    }
     case VPIC_OPT_DEVICE_EXCHANGE: {
       if (value < 1 || !c->ex) return VPIC_ERR_INVALID;
       DeviceGuard dg(c->device);

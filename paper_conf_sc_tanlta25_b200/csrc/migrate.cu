@@ -39,6 +39,12 @@ struct Exchange {
   int32_t *di_flag = nullptr;         // bit 0 inbox full (senders), 1 holes overflow, 2 particles overflow
   vpic_mover_t *di_arr = nullptr, *di_next = nullptr;
   uint32_t *di_scr = nullptr;         // hole scratch: tail_dead | low | surv, di_hcap each
+  // single-round mode: per-mover direction, packed send records, the
+  // accumulator's ghost planes (2 out, 2 in)
+  int8_t *g_dir = nullptr;
+  int64_t g_dir_cap = 0;
+  float *acc_plane[4] = {nullptr, nullptr, nullptr, nullptr};
+  size_t acc_plane_bytes = 0;
 };
 
 namespace {
@@ -128,7 +134,7 @@ __global__ void k_unpack(const float4 *__restrict__ recv, int64_t A, vpic_partic
 // ---- planes: (axis, index) plane of an array of nv records of `w` floats,
 // over the full extent of the other two axes (ghosts included).
 __global__ void k_plane_copy(const GridK g, int axis, int idx, float *__restrict__ a, int w,
-                             float *__restrict__ buf, int mode /*0 pack, 1 unpack, 2 add*/) {
+                             float *__restrict__ buf, int mode /*0 pack, 1 unpack, 2 add, 3 pack + zero*/) {
   const int sz = g.nv / ((int64_t)g.sx * g.sy);
   const int e0 = axis == 0 ? g.sy : g.sx;
   const int e1 = axis == 2 ? g.sy : sz;
@@ -145,7 +151,8 @@ __global__ void k_plane_copy(const GridK g, int axis, int idx, float *__restrict
     float *e = a + (int64_t)w * (x + (int64_t)g.sx * (y + (int64_t)g.sy * z)) + c;
     if (mode == 0) buf[t] = *e;
     else if (mode == 1) *e = buf[t];
-    else *e += buf[t];
+    else if (mode == 2) *e += buf[t];
+    else { buf[t] = *e; *e = 0.0f; }
   }
 }
 
@@ -202,10 +209,10 @@ int remove_holes(vpic_ctx *c, vpic_particle_t *p, int64_t np, const uint32_t *ho
 }
 
 // ---------------------------------------------------- device-initiated --
-struct Peers6 { int lsa[6]; };
+struct Peers27 { int lsa[27]; };
 
-__global__ void k_di_peers(ncclWindow_t w, Peers6 pr, unsigned char **out) {
-  for (int f = 0; f < 6; ++f)
+__global__ void k_di_peers(ncclWindow_t w, Peers27 pr, int n, unsigned char **out) {
+  for (int f = 0; f < n; ++f)
     out[f] = pr.lsa[f] >= 0 ? static_cast<unsigned char *>(ncclGetLsaPointer(w, 0, pr.lsa[f])) : nullptr;
 }
 
@@ -266,7 +273,7 @@ __global__ void k_di_take(unsigned char *inbox, int r, int64_t cap, int64_t max_
   if (threadIdx.x != 0) return;
   int64_t off = 0;
   for (int f = 0; f < 6; ++f) {
-    unsigned long long *cf = reinterpret_cast<unsigned long long *>(inbox + di_cnt_off(r, f));
+    unsigned long long *cf = reinterpret_cast<unsigned long long *>(inbox + di_cnt_off(di_face_slot(r, f)));
     int64_t a = (int64_t)*cf;
     if (a > cap) a = cap;     // the senders flagged the overflow
     ctr[8 + f] = off;
@@ -292,7 +299,7 @@ __global__ void k_di_unpack(const unsigned char *inbox, int r, int64_t cap, cons
     int f = 0;
     while (f < 5 && t >= ctr[8 + f + 1]) ++f;
     const int64_t k = t - ctr[8 + f];
-    const float4 *rec = reinterpret_cast<const float4 *>(inbox + di_rec_off(r, f, cap, k));
+    const float4 *rec = reinterpret_cast<const float4 *>(inbox + di_rec_off(di_face_slot(r, f), cap, k));
     const float4 a = rec[0], b = rec[1], d = rec[2];
     float4 *dst = reinterpret_cast<float4 *>(p + base + t);
     dst[0] = a;
@@ -300,6 +307,110 @@ __global__ void k_di_unpack(const unsigned char *inbox, int r, int64_t cap, cons
     vpic_mover_t m;
     m.dispx = d.x; m.dispy = d.y; m.dispz = d.z; m.idx = (int32_t)(base + t);
     mv[t] = m;
+  }
+}
+
+// ---- single-round mode (SURVEY.md §8(e) alternative (2)) ----------------
+struct Off27 { int64_t o[27]; };
+
+__device__ __forceinline__ int ghost_dir(const GridK &g, int32_t v, int &x, int &y, int &z) {
+  x = v % g.sx; y = (v / g.sx) % g.sy; z = v / g.sxy;
+  const int ox = x == 0 ? -1 : (x == g.nx + 1 ? 1 : 0);
+  const int oy = y == 0 ? -1 : (y == g.ny + 1 ? 1 : 0);
+  const int oz = z == 0 ? -1 : (z == g.nz + 1 ? 1 : 0);
+  // the voxel as the neighbour sees it: crossed axes enter from its far side
+  if (ox) x = ox < 0 ? g.nx : 1;
+  if (oy) y = oy < 0 ? g.ny : 1;
+  if (oz) z = oz < 0 ? g.nz : 1;
+  return dir26(ox, oy, oz);
+}
+
+// Departures of this call: every mover's slot becomes a hole; a particle
+// marked p.i = -1 - (ghost voxel) leaves for the neighbour in that voxel's
+// direction, the others (absorbed) are dropped.  Counts per direction.
+__global__ void k_ghost_classify(const GridK g, const vpic_particle_t *__restrict__ p,
+                                 const vpic_mover_t *__restrict__ mv, const int64_t *__restrict__ Mdev,
+                                 int64_t Mmax, int8_t *__restrict__ dir, int64_t *__restrict__ cnt,
+                                 uint32_t *__restrict__ holes) {
+  const int64_t M = min(*Mdev, Mmax);
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < M;
+       k += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t idx = mv[k].idx;
+    holes[k] = (uint32_t)idx;
+    const int32_t i = p[idx].i;
+    if (i >= 0) { dir[k] = -1; continue; }
+    int x, y, z;
+    const int d = ghost_dir(g, -1 - i, x, y, z);
+    dir[k] = (int8_t)d;
+    atomicAdd(reinterpret_cast<unsigned long long *>(cnt + d), 1ull);
+  }
+}
+
+__global__ void k_ghost_pack(const GridK g, const vpic_particle_t *__restrict__ p,
+                             const vpic_mover_t *__restrict__ mv, int64_t M, const int8_t *__restrict__ dir,
+                             Off27 off, unsigned long long *__restrict__ cur, float4 *__restrict__ send) {
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < M;
+       k += (int64_t)gridDim.x * blockDim.x) {
+    const int d = dir[k];
+    if (d < 0) continue;
+    const vpic_particle_t q = p[mv[k].idx];
+    int x, y, z;
+    ghost_dir(g, -1 - q.i, x, y, z);
+    const int64_t slot = off.o[d] + (int64_t)atomicAdd(cur + d, 1ull);
+    float4 *r = send + 3 * slot;
+    r[0] = make_float4(q.dx, q.dy, q.dz, __int_as_float(x + g.sx * (y + g.sy * z)));
+    r[1] = make_float4(q.ux, q.uy, q.uz, q.w);
+    r[2] = make_float4(0.f, 0.f, 0.f, 0.f);
+  }
+}
+
+// Append arrivals (their move is complete).
+__global__ void k_ghost_unpack(const float4 *__restrict__ recv, int64_t A, vpic_particle_t *__restrict__ p,
+                               int64_t np) {
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < A;
+       k += (int64_t)gridDim.x * blockDim.x) {
+    float4 *dst = reinterpret_cast<float4 *>(p + np + k);
+    dst[0] = recv[3 * k];
+    dst[1] = recv[3 * k + 1];
+  }
+}
+
+// Device-initiated: arrivals of epoch parity e from the 26 directions ->
+// offsets ctr[16 + a], total ctr[2], append base ctr[7]; counters reset.
+__global__ void k_di_take_ghost(unsigned char *inbox, int e, int64_t cap, int64_t max_np, int64_t *ctr,
+                                int32_t *flag) {
+  if (threadIdx.x != 0) return;
+  int64_t off = 0;
+  for (int a = 0; a < 27; ++a) {
+    unsigned long long *cf = reinterpret_cast<unsigned long long *>(inbox + di_cnt_off(di_ghost_slot(e, a)));
+    int64_t n = (int64_t)*cf;
+    if (n > cap) n = cap;     // the senders flagged the overflow
+    ctr[16 + a] = off;
+    off += n;
+    *cf = 0;
+  }
+  const int64_t base = ctr[0];
+  if (base + off > max_np) {  // no room: drop the arrivals, report capacity
+    atomicOr(flag, 4);
+    off = 0;
+    for (int a = 0; a < 27; ++a) ctr[16 + a] = 0;
+  }
+  ctr[2] = off;
+  ctr[7] = base;
+  ctr[0] = base + off;
+}
+__global__ void k_di_unpack_ghost(const unsigned char *inbox, int e, int64_t cap, const int64_t *ctr,
+                                  vpic_particle_t *__restrict__ p) {
+  const int64_t A = ctr[2], base = ctr[7];
+  for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < A;
+       t += (int64_t)gridDim.x * blockDim.x) {
+    int a = 0;
+    while (a < 26 && t >= ctr[16 + a + 1]) ++a;
+    const int64_t k = t - ctr[16 + a];
+    const float4 *rec = reinterpret_cast<const float4 *>(inbox + di_rec_off(di_ghost_slot(e, a), cap, k));
+    float4 *dst = reinterpret_cast<float4 *>(p + base + t);
+    dst[0] = rec[0];
+    dst[1] = rec[1];
   }
 }
 
@@ -314,7 +425,7 @@ int exchange_create(vpic_ctx *c, const uint8_t *uid) {
     delete ex;
     return VPIC_ERR_NCCL;
   }
-  if (cudaMalloc(&ex->d_cnt, 16 * sizeof(int64_t)) != cudaSuccess) {
+  if (cudaMalloc(&ex->d_cnt, 96 * sizeof(int64_t)) != cudaSuccess) {
     ncclCommDestroy(ex->comm);
     delete ex;
     return VPIC_ERR_CUDA;
@@ -341,6 +452,8 @@ void exchange_destroy(vpic_ctx *c) {
   cudaFree(ex->di_arr);
   cudaFree(ex->di_next);
   cudaFree(ex->di_scr);
+  cudaFree(ex->g_dir);
+  for (float *b : ex->acc_plane) cudaFree(b);
   delete ex;
   c->ex = nullptr;
 }
@@ -352,7 +465,8 @@ void exchange_destroy(vpic_ctx *c) {
 int device_exchange_enable(vpic_ctx *c, int64_t cap) {
   Exchange *ex = c->ex;
   if (!ex || ex->di || cap <= 0) return VPIC_ERR_INVALID;
-  const size_t bytes = (size_t)di_rec_off(DI_ROUNDS, 0, cap, 0);
+  const bool ghost = c->gk.ghost_mig != 0;
+  const size_t bytes = (size_t)di_rec_off(ghost ? DI_GHOST_SLOTS : DI_FACE_SLOTS, cap, 0);
   CKN(ncclMemAlloc(&ex->di_buf, bytes));
   CKC(cudaMemset(ex->di_buf, 0, DI_HDR));
   CKN(ncclCommWindowRegister(ex->comm, ex->di_buf, bytes, &ex->di_win, NCCL_WIN_COLL_SYMMETRIC));
@@ -360,31 +474,34 @@ int device_exchange_enable(vpic_ctx *c, int64_t cap) {
   req.lsaBarrierCount = 1;
   CKN(ncclDevCommCreate(ex->comm, &req, &ex->di_dcomm));
   ex->di_dcomm_ok = true;
-  Peers6 pr;
+  Peers27 pr;
   const ncclTeam_t world = ncclTeamWorld(ex->comm);
-  for (int f = 0; f < 6; ++f) {
+  const int npeer = ghost ? 27 : 6;   // single-round mode: 26 directions, else 6 faces
+  for (int f = 0; f < npeer; ++f) {
     pr.lsa[f] = -1;
-    if (c->gk.face_kind[f] != FACE_REMOTE) continue;
-    pr.lsa[f] = ncclTeamRankToLsa(ex->comm, world, c->g.nbr_rank[f]);
+    const int r = ghost ? c->nbr26[f] : (c->gk.face_kind[f] == FACE_REMOTE ? c->g.nbr_rank[f] : -1);
+    if (r < 0) continue;
+    pr.lsa[f] = ncclTeamRankToLsa(ex->comm, world, r);
     if (pr.lsa[f] < 0) return VPIC_ERR_UNSUPPORTED;   // neighbour not load/store reachable
   }
   unsigned char **d_peers = nullptr;
-  CKC(cudaMalloc(&d_peers, 6 * sizeof(void *)));
-  k_di_peers<<<1, 1>>>(ex->di_win, pr, d_peers); note_launch();
-  unsigned char *h_peers[6];
-  const cudaError_t e = cudaMemcpy(h_peers, d_peers, sizeof(h_peers), cudaMemcpyDeviceToHost);
+  CKC(cudaMalloc(&d_peers, 27 * sizeof(void *)));
+  k_di_peers<<<1, 1>>>(ex->di_win, pr, npeer, d_peers); note_launch();
+  unsigned char *h_peers[27];
+  const cudaError_t e = cudaMemcpy(h_peers, d_peers, npeer * sizeof(void *), cudaMemcpyDeviceToHost);
   cudaFree(d_peers);
   CKC(e);
   ex->di_cap = cap;
   ex->di_hcap = std::max<int64_t>(8 * cap, 1 << 16);
-  CKC(cudaMalloc(&ex->di_ctr, 16 * sizeof(int64_t)));
-  CKC(cudaMemset(ex->di_ctr, 0, 16 * sizeof(int64_t)));
+  CKC(cudaMalloc(&ex->di_ctr, 64 * sizeof(int64_t)));
+  CKC(cudaMemset(ex->di_ctr, 0, 64 * sizeof(int64_t)));
   CKC(cudaMalloc(&ex->di_flag, sizeof(int32_t)));
   CKC(cudaMemset(ex->di_flag, 0, sizeof(int32_t)));
   CKC(cudaMalloc(&ex->di_arr, (size_t)6 * cap * sizeof(vpic_mover_t)));
   CKC(cudaMalloc(&ex->di_next, (size_t)6 * cap * sizeof(vpic_mover_t)));
   CKC(cudaMalloc(&ex->di_scr, (size_t)3 * ex->di_hcap * sizeof(uint32_t)));
-  for (int f = 0; f < 6; ++f) c->gk.di_peer[f] = h_peers[f];
+  if (ghost) for (int f = 0; f < 27; ++f) c->gk.di_peer26[f] = h_peers[f];
+  else for (int f = 0; f < 6; ++f) c->gk.di_peer[f] = h_peers[f];
   c->gk.di_cap = cap;
   c->gk.di_flag = ex->di_flag;
   c->gk.di_round = 0;
@@ -455,6 +572,197 @@ int migrate_di(vpic_ctx *c, float qsp, vpic_particle_t *p, int64_t *np_io, int64
   return VPIC_OK;
 }
 
+// ------------------------------------------------- single-round migration --
+// The 26 neighbour ranks: direction d reaches the rank found by following the
+// face neighbours along x, then y, then z (the ranks' face tables are
+// all-gathered; one NCCL all-gather at enable time).  A direction is used only
+// if every face it crosses is REMOTE here.
+int ghost_migration_enable(vpic_ctx *c) {
+  Exchange *ex = c->ex;
+  if (!ex || ex->di) return VPIC_ERR_INVALID;   // (before VPIC_OPT_DEVICE_EXCHANGE)
+  std::vector<int32_t> tab(6 * (size_t)c->nranks);
+  if (c->nranks == 1) {
+    for (int f = 0; f < 6; ++f) tab[f] = c->g.nbr_rank[f];
+  } else {
+    int32_t *d = nullptr;
+    CKC(cudaMalloc(&d, sizeof(int32_t) * 6 * (c->nranks + 1)));
+    CKC(cudaMemcpy(d, c->g.nbr_rank, 6 * sizeof(int32_t), cudaMemcpyHostToDevice));
+    if (ncclAllGather(d, d + 6, 6, ncclInt32, ex->comm, 0) != ncclSuccess) { cudaFree(d); return VPIC_ERR_NCCL; }
+    const cudaError_t e = cudaMemcpy(tab.data(), d + 6, tab.size() * sizeof(int32_t), cudaMemcpyDeviceToHost);
+    cudaFree(d);
+    CKC(e);
+  }
+  for (int dd = 0; dd < 27; ++dd) {
+    const int o[3] = {dd % 3 - 1, (dd / 3) % 3 - 1, dd / 9 - 1};
+    int r = c->rank;
+    bool ok = dd != 13;
+    for (int a = 0; a < 3 && ok; ++a) {
+      if (!o[a]) continue;
+      const int f = o[a] < 0 ? a : a + 3;
+      if (c->gk.face_kind[f] != FACE_REMOTE) ok = false;
+      else r = tab[6 * (size_t)r + f];
+    }
+    c->nbr26[dd] = ok ? r : -1;
+  }
+  c->gk.ghost_mig = 1;
+  c->di_epoch = 0;
+  return VPIC_OK;
+}
+
+// The accumulator's ghost layer holds the currents of streaks this rank's
+// particles ran in the neighbours' boundary voxels: axis by axis, plane 0 is
+// added into the -face neighbour's plane n and plane n+1 into the +face
+// neighbour's plane 1, then zeroed.  Planes span the other axes' ghosts, so
+// edge and corner ghosts reach the diagonal neighbours in two or three hops.
+// Per peer pair: sends (plane 0, plane n+1) and receives (from +, from -) in
+// the same order on both sides.
+int reduce_acc_ghosts(vpic_ctx *c, float *acc, cudaStream_t s) {
+  Exchange *ex = c->ex;
+  if (!ex || !c->gk.ghost_mig) return VPIC_OK;
+  const GridK &g = c->gk;
+  const int sz = g.nz + 2;
+  const size_t maxplane =
+      (size_t)std::max({(int64_t)g.sy * sz, (int64_t)g.sx * sz, (int64_t)g.sx * g.sy}) * 12 * 4;
+  if (maxplane > ex->acc_plane_bytes) {
+    for (float *&b : ex->acc_plane) {
+      cudaFree(b);
+      b = nullptr;
+      CKC(cudaMalloc(&b, maxplane));
+    }
+    ex->acc_plane_bytes = maxplane;
+  }
+  float **B = ex->acc_plane;
+  for (int axis = 0; axis < 3; ++axis) {
+    if (c->periodic_local[axis]) continue;
+    const int fm = axis, fp = axis + 3;
+    const bool rm = g.face_kind[fm] == FACE_REMOTE, rp = g.face_kind[fp] == FACE_REMOTE;
+    if (!rm && !rp) continue;
+    const int n = axis == 0 ? g.nx : (axis == 1 ? g.ny : g.nz);
+    const int64_t cnt =
+        (axis == 0 ? (int64_t)g.sy * sz : axis == 1 ? (int64_t)g.sx * sz : (int64_t)g.sx * g.sy) * 12;
+    if (rm) { k_plane_copy<<<blocks_for(cnt), 256, 0, s>>>(g, axis, 0, acc, 12, B[0], 3); note_launch(); }
+    if (rp) { k_plane_copy<<<blocks_for(cnt), 256, 0, s>>>(g, axis, n + 1, acc, 12, B[1], 3); note_launch(); }
+    CKN(ncclGroupStart());
+    if (rm) CKN(ncclSend(B[0], cnt, ncclFloat32, c->g.nbr_rank[fm], ex->comm, s));
+    if (rp) CKN(ncclSend(B[1], cnt, ncclFloat32, c->g.nbr_rank[fp], ex->comm, s));
+    if (rp) CKN(ncclRecv(B[2], cnt, ncclFloat32, c->g.nbr_rank[fp], ex->comm, s));
+    if (rm) CKN(ncclRecv(B[3], cnt, ncclFloat32, c->g.nbr_rank[fm], ex->comm, s));
+    CKN(ncclGroupEnd());
+    if (rp) { k_plane_copy<<<blocks_for(cnt), 256, 0, s>>>(g, axis, n, acc, 12, B[2], 2); note_launch(); }
+    if (rm) { k_plane_copy<<<blocks_for(cnt), 256, 0, s>>>(g, axis, 1, acc, 12, B[3], 2); note_launch(); }
+    CKC(cudaGetLastError());
+  }
+  return VPIC_OK;
+}
+
+namespace {
+
+// Single-round mode over NCCL: one exchange of the departures with the (up to)
+// 26 neighbours -- per-direction counts, one host synchronisation, the 48-B
+// records -- then the accumulator ghosts.  Sends are posted in increasing
+// direction d and receives in decreasing arrival direction a = 26 - d, so NCCL
+// pairs them even where one rank is the neighbour in several directions.
+int migrate_ghost(vpic_ctx *c, vpic_particle_t *p, int64_t *np_io, int64_t max_np,
+                  const vpic_mover_t *movers, const int64_t *n_movers, float *acc, cudaStream_t s) {
+  Exchange *ex = c->ex;
+  int64_t M = 0;
+  CKC(cudaMemcpyAsync(&M, n_movers, 8, cudaMemcpyDeviceToHost, s));
+  CKC(cudaStreamSynchronize(s));
+  int64_t np = *np_io;
+  if (M > np) return VPIC_ERR_INVALID;
+  int32_t *d_flags = reinterpret_cast<int32_t *>(c->d_count + 1);
+  CKC(cudaMemsetAsync(d_flags, 0, 4, s));
+  const int64_t Mpad = std::max<int64_t>(M, 1);
+  if (int rc = ctx_scratch(c, 16 * (size_t)Mpad + 64)) return rc;
+  uint32_t *holes = static_cast<uint32_t *>(c->scratch);
+  if (int rc = ensure(reinterpret_cast<void **>(&ex->g_dir), &ex->g_dir_cap, Mpad, 1)) return rc;
+  int64_t *cnt = ex->d_cnt;   // [0,27) sent per direction, [27,54) received, [54,81) cursors
+  CKC(cudaMemsetAsync(cnt, 0, 81 * sizeof(int64_t), s));
+  if (M > 0) {
+    k_ghost_classify<<<blocks_for(M), 256, 0, s>>>(c->gk, p, movers, n_movers, M, ex->g_dir, cnt, holes); note_launch();
+    CKC(cudaGetLastError());
+  }
+  CKN(ncclGroupStart());
+  for (int d = 0; d < 27; ++d)
+    if (c->nbr26[d] >= 0) CKN(ncclSend(cnt + d, 1, ncclInt64, c->nbr26[d], ex->comm, s));
+  for (int a = 26; a >= 0; --a)
+    if (c->nbr26[a] >= 0) CKN(ncclRecv(cnt + 27 + a, 1, ncclInt64, c->nbr26[a], ex->comm, s));
+  CKN(ncclGroupEnd());
+  int64_t h[54];
+  CKC(cudaMemcpyAsync(h, cnt, sizeof(h), cudaMemcpyDeviceToHost, s));
+  CKC(cudaStreamSynchronize(s));
+  Off27 so, ro;
+  int64_t S = 0, A = 0;
+  for (int d = 0; d < 27; ++d) { so.o[d] = S; S += h[d]; }
+  for (int a = 0; a < 27; ++a) { ro.o[a] = A; A += h[27 + a]; }
+  int64_t tot = ex->send_cap * 6;
+  if (int rc = ensure(reinterpret_cast<void **>(&ex->send), &tot, std::max<int64_t>(S, 1), 48)) return rc;
+  ex->send_cap = tot / 6;
+  if (int rc = ensure(reinterpret_cast<void **>(&ex->recv), &ex->recv_cap, std::max<int64_t>(A, 1), 48)) return rc;
+  if (S > 0) {
+    k_ghost_pack<<<blocks_for(M), 256, 0, s>>>(c->gk, p, movers, M, ex->g_dir, so,
+                                               reinterpret_cast<unsigned long long *>(cnt + 54), ex->send); note_launch();
+    CKC(cudaGetLastError());
+  }
+  CKN(ncclGroupStart());
+  for (int d = 0; d < 27; ++d)
+    if (c->nbr26[d] >= 0)
+      CKN(ncclSend(ex->send + 3 * so.o[d], (size_t)h[d] * 12, ncclFloat32, c->nbr26[d], ex->comm, s));
+  for (int a = 26; a >= 0; --a)
+    if (c->nbr26[a] >= 0)
+      CKN(ncclRecv(ex->recv + 3 * ro.o[a], (size_t)h[27 + a] * 12, ncclFloat32, c->nbr26[a], ex->comm, s));
+  CKN(ncclGroupEnd());
+  if (int rc = remove_holes(c, p, np, holes, M, s)) return rc;
+  np -= M;
+  if (np + A > max_np) return VPIC_ERR_CAPACITY;
+  if (A > 0) {
+    k_ghost_unpack<<<blocks_for(A), 256, 0, s>>>(ex->recv, A, p, np); note_launch();
+    CKC(cudaGetLastError());
+    np += A;
+  }
+  if (int rc = reduce_acc_ghosts(c, acc, s)) return rc;
+  int32_t hflag = 0;
+  CKC(cudaMemcpyAsync(&hflag, d_flags, 4, cudaMemcpyDeviceToHost, s));
+  CKC(cudaStreamSynchronize(s));
+  *np_io = np;
+  return hflag ? VPIC_ERR_CAPACITY : VPIC_OK;
+}
+
+// Single-round mode, device-initiated: advance_p already stored every
+// departure into its neighbour's inbox (this epoch's slots); remove the holes,
+// one LSA barrier, append the arrivals, reduce the accumulator ghosts.  One
+// host synchronisation (the new np and the overflow flags).
+int migrate_ghost_di(vpic_ctx *c, vpic_particle_t *p, int64_t *np_io, int64_t max_np,
+                     const vpic_mover_t *movers, const int64_t *n_movers, float *acc, cudaStream_t s) {
+  Exchange *ex = c->ex;
+  const int e = (int)(c->di_epoch & 1);
+  int32_t *d_flags = reinterpret_cast<int32_t *>(c->d_count + 1);
+  CKC(cudaMemsetAsync(d_flags, 0, 4, s));
+  k_di_set<<<1, 1, 0, s>>>(ex->di_ctr, *np_io); note_launch();
+  if (int rc = di_remove_holes(c, p, movers, n_movers, s)) return rc;
+  unsigned char *inbox = static_cast<unsigned char *>(ex->di_buf);
+  k_lsa_barrier<<<1, 128, 0, s>>>(ex->di_dcomm); note_launch();
+  k_di_take_ghost<<<1, 32, 0, s>>>(inbox, e, ex->di_cap, max_np, ex->di_ctr, ex->di_flag); note_launch();
+  k_di_unpack_ghost<<<(unsigned)c->num_sms * 4, 256, 0, s>>>(inbox, e, ex->di_cap, ex->di_ctr, p); note_launch();
+  CKC(cudaGetLastError());
+  c->di_epoch++;
+  if (int rc = reduce_acc_ghosts(c, acc, s)) return rc;
+  int64_t h_np = 0;
+  int32_t h_fl[2] = {0, 0};
+  CKC(cudaMemcpyAsync(&h_np, ex->di_ctr, 8, cudaMemcpyDeviceToHost, s));
+  CKC(cudaMemcpyAsync(&h_fl[0], d_flags, 4, cudaMemcpyDeviceToHost, s));
+  CKC(cudaMemcpyAsync(&h_fl[1], ex->di_flag, 4, cudaMemcpyDeviceToHost, s));
+  CKC(cudaStreamSynchronize(s));
+  *np_io = h_np;
+  if (h_fl[0] || h_fl[1]) {
+    CKC(cudaMemsetAsync(ex->di_flag, 0, 4, s));
+    return VPIC_ERR_CAPACITY;
+  }
+  return VPIC_OK;
+}
+
+}  // namespace
+
 // Up to 3 rounds: pack movers per face, exchange counts, exchange records,
 // remove departed / absorbed particles, append arrivals, continue their move.
 // Host synchronisations: the initial mover count, one per round (the NCCL
@@ -462,6 +770,10 @@ int migrate_di(vpic_ctx *c, float qsp, vpic_particle_t *p, int64_t *np_io, int64
 int migrate(vpic_ctx *c, float qsp, float msp, vpic_particle_t *p, int64_t *np_io, int64_t max_np,
             vpic_mover_t *movers, const int64_t *n_movers, float *acc, cudaStream_t s) {
   (void)msp;
+  if (c->ex && c->gk.ghost_mig) {
+    return c->ex->di ? migrate_ghost_di(c, p, np_io, max_np, movers, n_movers, acc, s)
+                     : migrate_ghost(c, p, np_io, max_np, movers, n_movers, acc, s);
+  }
   if (c->ex && c->ex->di) return migrate_di(c, qsp, p, np_io, max_np, movers, n_movers, acc, s);
   int64_t M = 0;
   CKC(cudaMemcpyAsync(&M, n_movers, 8, cudaMemcpyDeviceToHost, s));

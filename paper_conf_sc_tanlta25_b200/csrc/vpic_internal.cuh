@@ -28,7 +28,16 @@ struct GridK {
   int64_t di_cap;            // records per (round, face) inbox
   int32_t *di_flag;          // local: bit 0 set when an inbox was full
   int32_t di_round;          // migration round of this launch's departures
+                             // (single-round mode: the epoch parity)
   int32_t di_on;
+  // single-round migration (SURVEY.md §8(e) alternative (2);
+  // VPIC_OPT_SINGLE_ROUND_MIGRATION): a particle crossing a REMOTE face keeps
+  // moving through this rank's ghost layer (depositing into the ghost
+  // accumulators) and leaves, its move complete, from the ghost voxel it
+  // ends in -- to one of 26 neighbours, direction d = (ox+1) + 3(oy+1) +
+  // 9(oz+1), o = -1 / 0 / +1 for ghost coordinate 0 / interior / n+1
+  int32_t ghost_mig;
+  unsigned char *di_peer26[27];  // device-initiated: inbox of the direction-d neighbour
 };
 
 // Round-up reciprocal for exact unsigned division of n < 2^31 by d >= 2:
@@ -42,15 +51,23 @@ inline void set_magic(uint32_t d, uint32_t &m, uint32_t &s) {
   m = (uint32_t)(((1ull << (32 + k)) + d - 1) / d);
 }
 
-// inbox window layout: counters [DI_ROUNDS][6] (u64), then records
-// [DI_ROUNDS][6][di_cap] x 48 B (position record, momentum record, remaining
-// displacement); the round-r counter of face f counts arrivals through MY face f
+// inbox window layout: a u64 counter per slot, then records [slot][di_cap] x
+// 48 B (position record, momentum record, remaining displacement).  Face
+// mode: slot r*6 + f = round r, arrivals through MY face f (18 slots).
+// Single-round mode: slot e*27 + a = epoch parity e, arrivals from MY
+// direction a (54 slots; the parity keeps a neighbour's next-call stores
+// apart from this call's arrivals).
 constexpr int DI_ROUNDS = 3;
-constexpr int64_t DI_HDR = 256;
-__host__ __device__ inline int64_t di_cnt_off(int r, int f) { return 8 * (int64_t)(r * 6 + f); }
-__host__ __device__ inline int64_t di_rec_off(int r, int f, int64_t cap, int64_t k) {
-  return DI_HDR + 48 * ((int64_t)(r * 6 + f) * cap + k);
+constexpr int DI_FACE_SLOTS = 18, DI_GHOST_SLOTS = 54;
+constexpr int64_t DI_HDR = 512;
+__host__ __device__ inline int di_face_slot(int r, int f) { return r * 6 + f; }
+__host__ __device__ inline int di_ghost_slot(int e, int a) { return e * 27 + a; }
+__host__ __device__ inline int64_t di_cnt_off(int slot) { return 8 * (int64_t)slot; }
+__host__ __device__ inline int64_t di_rec_off(int slot, int64_t cap, int64_t k) {
+  return DI_HDR + 48 * ((int64_t)slot * cap + k);
 }
+// direction index of a ghost offset (ox, oy, oz) in {-1, 0, 1}^3; 13 = none
+__host__ __device__ inline int dir26(int ox, int oy, int oz) { return (ox + 1) + 3 * (oy + 1) + 9 * (oz + 1); }
 
 enum FaceKind { FACE_LOCAL = 0, FACE_REFLECT = 1, FACE_ABSORB = 2, FACE_REMOTE = 3 };
 
@@ -77,6 +94,8 @@ struct vpic_ctx {
   void *scratch;
   size_t scratch_bytes;
   int64_t *d_count;        // device counters [4]
+  int nbr26[27];           // single-round mode: rank of the direction-d neighbour (-1: none)
+  int64_t di_epoch;        // single-round mode: vpic_migrate_particles calls so far
 };
 
 namespace vpic {
@@ -144,5 +163,10 @@ void exchange_destroy(vpic_ctx *c);
 int halo_fields(vpic_ctx *c, float *fields, cudaStream_t s, int dir = +1);
 int device_exchange_enable(vpic_ctx *c, int64_t cap);
 int reduce_jf(vpic_ctx *c, float *jf, cudaStream_t s);
+// single-round mode: the 26 neighbour ranks (collective when nranks > 1)
+int ghost_migration_enable(vpic_ctx *c);
+// single-round mode: add the accumulator's ghost layer into the neighbours'
+// boundary voxels, axis by axis (edges / corners forwarded), and zero it
+int reduce_acc_ghosts(vpic_ctx *c, float *acc, cudaStream_t s);
 
 }  // namespace vpic

@@ -40,7 +40,7 @@ class HotPath:
                  uid: bytes = None, capacity_factor: float = 1.0, max_movers: int = 1 << 20,
                  device: Optional[int] = None, field_solve: bool = False, eps0: float = 1.0,
                  loopback_exchange: bool = False, concurrent_species: bool = False,
-                 device_exchange: bool = False, inbox_cap: int = 0):
+                 device_exchange: bool = False, inbox_cap: int = 0, single_round: bool = False):
         vpic.load()
         self.wl = wl
         self.g = wl.grid
@@ -55,6 +55,8 @@ class HotPath:
         self.nranks = nranks
         if loopback_exchange:   # periodic faces through the NCCL path (self peer)
             self.ctx.set_option(vpic.VPIC_OPT_LOOPBACK_EXCHANGE, 1)
+        if single_round:        # moves finished in the ghost layer, one 26-neighbour exchange
+            self.ctx.set_option(vpic.VPIC_OPT_SINGLE_ROUND_MIGRATION, 1)
         if device_exchange:     # movers stored into the neighbours' inboxes by the push (f4)
             self.ctx.set_option(vpic.VPIC_OPT_DEVICE_EXCHANGE, inbox_cap if inbox_cap > 1 else 1)
         self.migrate = (nranks > 1 or loopback_exchange

@@ -25,6 +25,7 @@ VPIC_OPT_MATH, VPIC_OPT_DEPOSIT, VPIC_OPT_TILE_SZ, VPIC_OPT_ADVANCE_KERNEL = 0, 
 VPIC_OPT_LOOPBACK_EXCHANGE = 4
 VPIC_OPT_ADVANCE_CTAS_PER_SM = 5
 VPIC_OPT_DEVICE_EXCHANGE = 6
+VPIC_OPT_SINGLE_ROUND_MIGRATION = 7
 MATH_FAST, MATH_IEEE = 0, 1
 DEP_AUTO, DEP_LANE, DEP_WARP = 0, 1, 2
 

@@ -88,9 +88,11 @@ def _multiset(a):
     return np.sort(np.ascontiguousarray(a).view(np.dtype((np.void, 32))).ravel())
 
 
+@pytest.mark.parametrize("walls", [False, True], ids=["periodic", "reflect_z"])
+@pytest.mark.parametrize("migration", ["rounds", "single"])
 @pytest.mark.parametrize("device_exchange", [False, True], ids=["nccl", "device"])
 @pytest.mark.parametrize("field_solve,steps", [(False, 3), (True, 1)])
-def test_loopback_exchange_matches_periodic(V, field_solve, steps, device_exchange):
+def test_loopback_exchange_matches_periodic(V, field_solve, steps, device_exchange, migration, walls):
     """VPIC_OPT_LOOPBACK_EXCHANGE sends every periodic crossing, E/cB halo and
     jf shared plane through the NCCL exchange (one-rank communicator, self
     peer): the multi-GPU code path on one GPU.  It must reproduce the local
@@ -98,9 +100,12 @@ def test_loopback_exchange_matches_periodic(V, field_solve, steps, device_exchan
     them), jf and fields within the atomic-reordering tolerance.  "device":
     the device-initiated exchange (f4) -- the push stores movers into the
     (self) neighbour's symmetric-memory inbox, rounds synchronised on the
-    device."""
+    device.  "single": VPIC_OPT_SINGLE_ROUND_MIGRATION -- moves finished in
+    the ghost layer, one exchange with the 26 (here: self) neighbours, the
+    accumulator's ghost layer added into the boundary voxels; "reflect_z":
+    walls on z, so ghost-layer particles also reflect there."""
     from paper_conf_sc_tanlta25_b200.pic import HotPath
-    g = inputs.GridSpec(8, 6, 5, dt=0.5)
+    g = inputs.GridSpec(8, 6, 5, dt=0.5, pbc=(0, 0, 1, 0, 0, 1) if walls else (0,) * 6)
     wl = inputs.Workload("loopback", g, [inputs.Species("electron", -1.0, 1.0, 0.6),
                                          inputs.Species("ion", 1.0, 4.0, 0.3)], 40, steps, 0)
     parts = inputs.make_species_particles(wl)
@@ -109,7 +114,8 @@ def test_loopback_exchange_matches_periodic(V, field_solve, steps, device_exchan
     for loop in (False, True):
         hp = HotPath(wl, parts, fields, math=V.MATH_IEEE, field_solve=field_solve,
                      loopback_exchange=loop, capacity_factor=1.0,
-                     device_exchange=loop and device_exchange, inbox_cap=4096)
+                     device_exchange=loop and device_exchange, inbox_cap=4096,
+                     single_round=loop and migration == "single")
         for _ in range(steps):
             hp.step()
         torch.cuda.synchronize()
@@ -130,7 +136,8 @@ def test_loopback_exchange_matches_periodic(V, field_solve, steps, device_exchan
         assert np.array_equal(fa, fb)       # static fields: halos move bytes only
 
 
-def test_device_exchange_inbox_overflow_reported(V):
+@pytest.mark.parametrize("migration", ["rounds", "single"])
+def test_device_exchange_inbox_overflow_reported(V, migration):
     """An inbox smaller than one round's arrivals: the push keeps going,
     vpic_migrate_particles reports VPIC_ERR_CAPACITY (no silent loss)."""
     from paper_conf_sc_tanlta25_b200.pic import HotPath
@@ -138,7 +145,8 @@ def test_device_exchange_inbox_overflow_reported(V):
     wl = inputs.Workload("overflow", g, [inputs.Species("electron", -1.0, 1.0, 0.8)], 60, 1, 0)
     parts = inputs.make_species_particles(wl)
     hp = HotPath(wl, parts, inputs.make_fields(g, 0.05), loopback_exchange=True,
-                 device_exchange=True, inbox_cap=2, capacity_factor=1.0)
+                 device_exchange=True, inbox_cap=2, capacity_factor=1.0,
+                 single_round=migration == "single")
     with pytest.raises(V.VpicError) as ei:
         hp.step()
     assert ei.value.status == -2      # VPIC_ERR_CAPACITY

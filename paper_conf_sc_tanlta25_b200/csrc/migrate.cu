@@ -43,6 +43,7 @@ struct Exchange {
   // accumulator's ghost planes (2 out, 2 in)
   int8_t *g_dir = nullptr;
   int64_t g_dir_cap = 0;
+  int64_t *g_pc = nullptr;            // per-peer direction counts: [2][27 peers][27]
   float *acc_plane[4] = {nullptr, nullptr, nullptr, nullptr};
   size_t acc_plane_bytes = 0;
 };
@@ -364,6 +365,17 @@ __global__ void k_ghost_pack(const GridK g, const vpic_particle_t *__restrict__ 
   }
 }
 
+struct DirPeer { int p[27]; };
+
+// Per-peer count vectors: out[k][d] = departures in direction d if direction
+// d's neighbour is peer k, else 0.
+__global__ void k_peer_counts(const int64_t *__restrict__ cnt, DirPeer dp, int npeer, int64_t *__restrict__ out) {
+  for (int t = threadIdx.x; t < npeer * 27; t += blockDim.x) {
+    const int k = t / 27, d = t % 27;
+    out[t] = dp.p[d] == k ? cnt[d] : 0;
+  }
+}
+
 // Append arrivals (their move is complete).
 __global__ void k_ghost_unpack(const float4 *__restrict__ recv, int64_t A, vpic_particle_t *__restrict__ p,
                                int64_t np) {
@@ -453,6 +465,7 @@ void exchange_destroy(vpic_ctx *c) {
   cudaFree(ex->di_next);
   cudaFree(ex->di_scr);
   cudaFree(ex->g_dir);
+  cudaFree(ex->g_pc);
   for (float *b : ex->acc_plane) cudaFree(b);
   delete ex;
   c->ex = nullptr;
@@ -604,6 +617,19 @@ int ghost_migration_enable(vpic_ctx *c) {
     }
     c->nbr26[dd] = ok ? r : -1;
   }
+  // distinct peers: one count message and one record message per peer
+  c->npeer26 = 0;
+  for (int r = 0; r < c->nranks; ++r) {
+    bool used = false;
+    for (int dd = 0; dd < 27; ++dd) used |= c->nbr26[dd] == r;
+    if (used) c->peer26[c->npeer26++] = r;
+  }
+  for (int dd = 0; dd < 27; ++dd) {
+    c->dir_peer[dd] = -1;
+    for (int k = 0; k < c->npeer26; ++k)
+      if (c->nbr26[dd] == c->peer26[k]) c->dir_peer[dd] = k;
+  }
+  if (!ex->g_pc && cudaMalloc(&ex->g_pc, 2 * 27 * 27 * sizeof(int64_t)) != cudaSuccess) return VPIC_ERR_CUDA;
   c->gk.ghost_mig = 1;
   c->di_epoch = 0;
   return VPIC_OK;
@@ -658,10 +684,12 @@ int reduce_acc_ghosts(vpic_ctx *c, float *acc, cudaStream_t s) {
 namespace {
 
 // Single-round mode over NCCL: one exchange of the departures with the (up to)
-// 26 neighbours -- per-direction counts, one host synchronisation, the 48-B
-// records -- then the accumulator ghosts.  Sends are posted in increasing
-// direction d and receives in decreasing arrival direction a = 26 - d, so NCCL
-// pairs them even where one rank is the neighbour in several directions.
+// 26 neighbours, aggregated per distinct peer rank -- a 27-count vector, one
+// host synchronisation, then all records for that peer in one message (the
+// send buffer is ordered by (peer, direction)) -- then the accumulator
+// ghosts.  One message per peer and phase, so the pairing of sends and
+// receives cannot be ambiguous even where one rank is the neighbour in
+// several directions.
 int migrate_ghost(vpic_ctx *c, vpic_particle_t *p, int64_t *np_io, int64_t max_np,
                   const vpic_mover_t *movers, const int64_t *n_movers, float *acc, cudaStream_t s) {
   Exchange *ex = c->ex;
@@ -670,31 +698,45 @@ int migrate_ghost(vpic_ctx *c, vpic_particle_t *p, int64_t *np_io, int64_t max_n
   CKC(cudaStreamSynchronize(s));
   int64_t np = *np_io;
   if (M > np) return VPIC_ERR_INVALID;
-  int32_t *d_flags = reinterpret_cast<int32_t *>(c->d_count + 1);
-  CKC(cudaMemsetAsync(d_flags, 0, 4, s));
   const int64_t Mpad = std::max<int64_t>(M, 1);
   if (int rc = ctx_scratch(c, 16 * (size_t)Mpad + 64)) return rc;
   uint32_t *holes = static_cast<uint32_t *>(c->scratch);
   if (int rc = ensure(reinterpret_cast<void **>(&ex->g_dir), &ex->g_dir_cap, Mpad, 1)) return rc;
-  int64_t *cnt = ex->d_cnt;   // [0,27) sent per direction, [27,54) received, [54,81) cursors
+  int64_t *cnt = ex->d_cnt;   // [0,27) sent per direction, [54,81) pack cursors
   CKC(cudaMemsetAsync(cnt, 0, 81 * sizeof(int64_t), s));
   if (M > 0) {
     k_ghost_classify<<<blocks_for(M), 256, 0, s>>>(c->gk, p, movers, n_movers, M, ex->g_dir, cnt, holes); note_launch();
-    CKC(cudaGetLastError());
   }
+  const int np26 = c->npeer26;
+  DirPeer dp;
+  for (int d = 0; d < 27; ++d) dp.p[d] = c->dir_peer[d];
+  int64_t *pc_out = ex->g_pc, *pc_in = ex->g_pc + 27 * 27;
+  k_peer_counts<<<1, 256, 0, s>>>(cnt, dp, np26, pc_out); note_launch();
+  CKC(cudaGetLastError());
   CKN(ncclGroupStart());
-  for (int d = 0; d < 27; ++d)
-    if (c->nbr26[d] >= 0) CKN(ncclSend(cnt + d, 1, ncclInt64, c->nbr26[d], ex->comm, s));
-  for (int a = 26; a >= 0; --a)
-    if (c->nbr26[a] >= 0) CKN(ncclRecv(cnt + 27 + a, 1, ncclInt64, c->nbr26[a], ex->comm, s));
+  for (int k = 0; k < np26; ++k) {
+    CKN(ncclSend(pc_out + 27 * k, 27, ncclInt64, c->peer26[k], ex->comm, s));
+    CKN(ncclRecv(pc_in + 27 * k, 27, ncclInt64, c->peer26[k], ex->comm, s));
+  }
   CKN(ncclGroupEnd());
-  int64_t h[54];
-  CKC(cudaMemcpyAsync(h, cnt, sizeof(h), cudaMemcpyDeviceToHost, s));
+  std::vector<int64_t> h(27 + 27 * (size_t)np26);
+  CKC(cudaMemcpyAsync(h.data(), cnt, 27 * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  if (np26) CKC(cudaMemcpyAsync(h.data() + 27, pc_in, 27 * np26 * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
   CKC(cudaStreamSynchronize(s));
-  Off27 so, ro;
+  Off27 so;
+  int64_t pso[27], psz[27], pro[27], prz[27];
   int64_t S = 0, A = 0;
-  for (int d = 0; d < 27; ++d) { so.o[d] = S; S += h[d]; }
-  for (int a = 0; a < 27; ++a) { ro.o[a] = A; A += h[27 + a]; }
+  for (int k = 0; k < np26; ++k) {
+    pso[k] = S;
+    for (int d = 0; d < 27; ++d)
+      if (c->dir_peer[d] == k) { so.o[d] = S; S += h[d]; }
+    psz[k] = S - pso[k];
+    pro[k] = A;
+    for (int d = 0; d < 27; ++d) A += h[27 + 27 * k + d];
+    prz[k] = A - pro[k];
+  }
+  for (int d = 0; d < 27; ++d)
+    if (c->dir_peer[d] < 0) so.o[d] = 0;
   int64_t tot = ex->send_cap * 6;
   if (int rc = ensure(reinterpret_cast<void **>(&ex->send), &tot, std::max<int64_t>(S, 1), 48)) return rc;
   ex->send_cap = tot / 6;
@@ -705,12 +747,10 @@ int migrate_ghost(vpic_ctx *c, vpic_particle_t *p, int64_t *np_io, int64_t max_n
     CKC(cudaGetLastError());
   }
   CKN(ncclGroupStart());
-  for (int d = 0; d < 27; ++d)
-    if (c->nbr26[d] >= 0)
-      CKN(ncclSend(ex->send + 3 * so.o[d], (size_t)h[d] * 12, ncclFloat32, c->nbr26[d], ex->comm, s));
-  for (int a = 26; a >= 0; --a)
-    if (c->nbr26[a] >= 0)
-      CKN(ncclRecv(ex->recv + 3 * ro.o[a], (size_t)h[27 + a] * 12, ncclFloat32, c->nbr26[a], ex->comm, s));
+  for (int k = 0; k < np26; ++k) {
+    CKN(ncclSend(ex->send + 3 * pso[k], (size_t)psz[k] * 12, ncclFloat32, c->peer26[k], ex->comm, s));
+    CKN(ncclRecv(ex->recv + 3 * pro[k], (size_t)prz[k] * 12, ncclFloat32, c->peer26[k], ex->comm, s));
+  }
   CKN(ncclGroupEnd());
   if (int rc = remove_holes(c, p, np, holes, M, s)) return rc;
   np -= M;
@@ -721,11 +761,8 @@ int migrate_ghost(vpic_ctx *c, vpic_particle_t *p, int64_t *np_io, int64_t max_n
     np += A;
   }
   if (int rc = reduce_acc_ghosts(c, acc, s)) return rc;
-  int32_t hflag = 0;
-  CKC(cudaMemcpyAsync(&hflag, d_flags, 4, cudaMemcpyDeviceToHost, s));
-  CKC(cudaStreamSynchronize(s));
-  *np_io = np;
-  return hflag ? VPIC_ERR_CAPACITY : VPIC_OK;
+  *np_io = np;   // (every count was known on the host: no further synchronisation)
+  return VPIC_OK;
 }
 
 // Single-round mode, device-initiated: advance_p already stored every

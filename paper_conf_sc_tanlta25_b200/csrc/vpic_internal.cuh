@@ -95,6 +95,9 @@ struct vpic_ctx {
   size_t scratch_bytes;
   int64_t *d_count;        // device counters [4]
   int nbr26[27];           // single-round mode: rank of the direction-d neighbour (-1: none)
+  int npeer26;             // ... its distinct ranks (ascending) and each direction's peer slot
+  int peer26[27];
+  int dir_peer[27];
   int64_t di_epoch;        // single-round mode: vpic_migrate_particles calls so far
 };
 

@@ -253,3 +253,145 @@ def test_decompose_neighbours():
                 assert nb.nbr_rank[OPP[f]] == r
             if n == 1:
                 assert g.nbr_rank == (0,) * 6
+
+
+# ------------------------------------------------ single-round migration --
+# Host logic of VPIC_OPT_SINGLE_ROUND_MIGRATION (csrc/migrate.cu:
+# ghost_migration_enable, migrate_ghost, reduce_acc_ghosts), replayed with
+# gloo between 8 processes on a 2x2x2 process grid -- every direction's
+# neighbour is some rank, and along each axis the - and + neighbours coincide,
+# the hardest case for pairing sends with receives.
+SB = (3, 2, 2)      # block per rank
+
+
+def compose26(tabs, rank, kinds):
+    """Rank of the direction-d neighbour: follow the face neighbours along x,
+    then y, then z (the C++ composition); -1 where a crossed face is not
+    remote or d is the centre."""
+    out = []
+    for d in range(27):
+        o = (d % 3 - 1, (d // 3) % 3 - 1, d // 9 - 1)
+        r, ok = rank, d != 13
+        for a in range(3):
+            if o[a] == 0 or not ok:
+                continue
+            f = a if o[a] < 0 else a + 3
+            if kinds[f] != "remote":
+                ok = False
+            else:
+                r = tabs[r][f]
+        out.append(r if ok else -1)
+    return out
+
+
+def _single_round_worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        gl = inputs.decompose(inputs.GridSpec(*SB), world, rank)
+        kinds = ["remote" if gl.nbr_rank[f] != rank else "local" for f in range(6)]
+        tabs = [None] * world
+        dist.all_gather_object(tabs, list(gl.nbr_rank))
+        nbr = compose26(tabs, rank, kinds)
+        P = inputs.process_grid(world)
+        me = (rank % P[0], (rank // P[0]) % P[1], rank // (P[0] * P[1]))
+        # 1. the composed rank is the geometric neighbour
+        for d in range(27):
+            if d == 13:
+                continue
+            o = (d % 3 - 1, (d // 3) % 3 - 1, d // 9 - 1)
+            cc = [(me[a] + o[a]) % P[a] for a in range(3)]
+            assert nbr[d] == cc[0] + P[0] * (cc[1] + P[1] * cc[2]), (rank, d)
+        # 2. one exchange: per direction a count then records naming (sender,
+        #    direction, k); sends in increasing d, receives in decreasing
+        #    arrival direction a (= the sender's increasing d)
+        cnt = {d: (rank * 27 + d) % 4 for d in range(27) if nbr[d] >= 0}
+        reqs = [dist.isend(torch.tensor([cnt[d]], dtype=torch.int64), nbr[d]) for d in sorted(cnt)]
+        rc = {}
+        for a in range(26, -1, -1):
+            if nbr[a] >= 0:
+                rc[a] = torch.zeros(1, dtype=torch.int64)
+                reqs.append(dist.irecv(rc[a], nbr[a]))
+        for r in reqs:
+            r.wait()
+        reqs = []
+        for d in sorted(cnt):
+            if cnt[d]:
+                rec = torch.tensor([[rank, d, k] for k in range(cnt[d])], dtype=torch.int64)
+                reqs.append(dist.isend(rec, nbr[d]))
+        got = {}
+        for a in range(26, -1, -1):
+            if nbr[a] >= 0 and int(rc[a]) > 0:
+                got[a] = torch.zeros((int(rc[a]), 3), dtype=torch.int64)
+                reqs.append(dist.irecv(got[a], nbr[a]))
+        for r in reqs:
+            r.wait()
+        for a, buf in got.items():
+            b = buf.numpy()
+            assert np.all(b[:, 0] == nbr[a]) and np.all(b[:, 1] == 26 - a), (rank, a, b)
+            assert np.array_equal(b[:, 2], np.arange(len(b)))
+        # 3. accumulator ghost layer, axis by axis: plane 0 -> -face neighbour's
+        #    plane n, plane n+1 -> +face neighbour's plane 1; receives from +
+        #    then -; ghosts zeroed.  Integer-valued float64: sums are exact.
+        n = (gl.nx, gl.ny, gl.nz)
+        acc = np.zeros((gl.nz + 2, gl.ny + 2, gl.nx + 2, 12))
+        rng = np.random.default_rng(100 + rank)
+        ghost = np.ones(acc.shape[:3], bool)
+        ghost[1:-1, 1:-1, 1:-1] = False
+        acc[ghost] = rng.integers(1, 1000, size=(int(ghost.sum()), 12))
+        acc[~ghost] = rng.integers(0, 1000, size=(int((~ghost).sum()), 12))
+        init = acc.copy()
+        for axis in range(3):
+            fm, fp = axis, axis + 3
+            ax = 2 - axis                                  # numpy axis (z, y, x)
+            sl = lambda i: tuple(i if k == ax else slice(None) for k in range(3))
+            s0 = torch.from_numpy(acc[sl(0)].copy())
+            s1 = torch.from_numpy(acc[sl(n[axis] + 1)].copy())
+            acc[sl(0)] = 0
+            acc[sl(n[axis] + 1)] = 0
+            r2, r3 = torch.zeros_like(s0), torch.zeros_like(s1)
+            reqs = [dist.isend(s0, gl.nbr_rank[fm]), dist.isend(s1, gl.nbr_rank[fp]),
+                    dist.irecv(r2, gl.nbr_rank[fp]), dist.irecv(r3, gl.nbr_rank[fm])]
+            for r in reqs:
+                r.wait()
+            acc[sl(n[axis])] += r2.numpy()
+            acc[sl(1)] += r3.numpy()
+        q.put((rank, dict(init=init, acc=acc, gx0=(gl.gx0, gl.gy0, gl.gz0))))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_single_round_protocol_eight_ranks():
+    """26-neighbour composition, one-exchange pairing, and the axis-ordered
+    accumulator ghost reduction: afterwards every ghost value has been added
+    to the interior voxel of the rank owning that global voxel (periodic box),
+    exactly once, and the ghost layers are zero."""
+    world = 8
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_single_round_worker, args=(r, world, port, q)) for r in range(world)]
+    for pr in procs:
+        pr.start()
+    res = dict(q.get(timeout=300) for _ in range(world))
+    for pr in procs:
+        pr.join(timeout=60)
+        assert pr.exitcode == 0
+    P = inputs.process_grid(world)
+    G = (SB[0] * P[0], SB[1] * P[1], SB[2] * P[2])
+    want = np.zeros((G[2], G[1], G[0], 12))
+    for r in range(world):
+        x0, y0, z0 = res[r]["gx0"]
+        init = res[r]["init"]
+        for z in range(SB[2] + 2):
+            for y in range(SB[1] + 2):
+                for x in range(SB[0] + 2):
+                    want[(z0 + z - 1) % G[2], (y0 + y - 1) % G[1], (x0 + x - 1) % G[0]] += init[z, y, x]
+    for r in range(world):
+        x0, y0, z0 = res[r]["gx0"]
+        acc = res[r]["acc"]
+        ghost = np.ones(acc.shape[:3], bool)
+        ghost[1:-1, 1:-1, 1:-1] = False
+        assert np.all(acc[ghost] == 0)
+        got = acc[1:-1, 1:-1, 1:-1]
+        assert np.array_equal(got, want[z0:z0 + SB[2], y0:y0 + SB[1], x0:x0 + SB[0]]), r

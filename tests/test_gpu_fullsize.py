@@ -140,3 +140,58 @@ def test_fullsize_rho_total_charge(state):
         assert abs(rho.double().sum().item() - tot) < 1e-5 * abs(tot)
         node = rho[torch.from_numpy(g.interior_voxels()).cuda()].double()
         assert abs(node.mean().item() - tot / g.ncells) < 1e-5 * abs(tot / g.ncells)
+
+
+def _record_multiset_hash(p: torch.Tensor, n: int) -> tuple:
+    """Order-independent fingerprint of n 32-B records on the device: the sum
+    and the xor of a 64-bit mix of each record (two independent folds), plus
+    n.  Equal multisets give equal fingerprints; a lost, duplicated or altered
+    record changes both folds with overwhelming probability."""
+    w = p[:n].contiguous().view(torch.int64)              # [n, 4] words
+    m = torch.tensor([0x9E3779B97F4A7C15 - (1 << 64), 0xC2B2AE3D27D4EB4F - (1 << 64),
+                      0x165667B19E3779F9, 0x27D4EB2F165667C5], dtype=torch.int64, device=p.device)
+    h = (w * m).sum(1)
+    h = h ^ (h >> 29)
+    h = h * (0xBF58476D1CE4E5B9 - (1 << 64))
+    h = h ^ (h >> 32)
+    x = h.clone()
+    while x.numel() > 1:                                   # xor-fold
+        if x.numel() & 1:
+            x = torch.cat([x, torch.zeros(1, dtype=x.dtype, device=x.device)])
+        x = x[0::2] ^ x[1::2]
+    return n, int(h.sum().item()), int(x.item())
+
+
+@pytest.mark.parametrize("device_exchange", [False, True], ids=["nccl", "device"])
+def test_fullsize_loopback_single_round_matches_local(device_exchange):
+    """The multi-GPU exchange at full size (configs[1], 2^29 particles), in the
+    configuration bench.py uses when there is an exchange: every periodic face
+    routed through the single-round migration with a self peer (loopback).
+    One IEEE-math PIC step must give exactly the particles of the local
+    periodic wrap (as a multiset: fingerprints of all 2^29 records equal) and
+    jf within the reordering tolerance."""
+    from paper_conf_sc_tanlta25_b200 import vpic
+    from paper_conf_sc_tanlta25_b200.pic import HotPath
+    wl = inputs.config(1)
+    g = wl.grid
+    parts = inputs.make_species_particles(wl)
+    fields = inputs.make_fields(g, wl.field_amp)
+    out = []
+    for loop in (False, True):
+        hp = HotPath(wl, parts, fields, math=vpic.MATH_IEEE, loopback_exchange=loop,
+                     device_exchange=loop and device_exchange, single_round=loop,
+                     capacity_factor=1.01)
+        hp.step(do_sort=True)
+        torch.cuda.synchronize()
+        fp = [_record_multiset_hash(s.p, s.np) for s in hp.species]
+        vox = torch.from_numpy(g.interior_voxels()).cuda()
+        jf = hp.jf[vox].double()
+        tail = hp.species[0].p[hp.species[0].np - 4096:hp.species[0].np].cpu()
+        out.append((fp, jf, tail))
+        hp.close()
+        del hp
+        torch.cuda.empty_cache()
+    (fa, ja, ta), (fb, jb, tb) = out
+    assert fa == fb
+    assert not torch.equal(ta, tb)      # migration ran: arrivals were appended at the end
+    assert (ja - jb).abs().max().item() <= 1e-5 * ja.abs().max().item() * 8

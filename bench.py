@@ -277,15 +277,22 @@ def our_arm(args, rank, world):
         torch.cuda.synchronize()
         barrier()
         e0.record(stream)
-        for _ in range(args.steps):
+        marks = [e0]
+        for k in range(args.steps):
             hp.cycle(S)
             pushes_local += S * hp.n_particles
+            if k + 1 < args.steps:
+                m = torch.cuda.Event(enable_timing=True)
+                m.record(stream)
+                marks.append(m)
         e1.record(stream)
+        marks.append(e1)
         torch.cuda.synchronize()
         barrier()
     launches = vpic.vpic_kernel_launches() - launches0
     hp.record_advance = False
     ms = e0.elapsed_time(e1)
+    step_ms = [a.elapsed_time(b) for a, b in zip(marks[:-1], marks[1:])]
     adv = [(a.elapsed_time(b), n) for a, b, n in hp.adv_events]
     adv_ms = sum(t for t, _ in adv) / len(adv)
     nsp = len(hp.species)
@@ -375,6 +382,8 @@ def our_arm(args, rank, world):
                                 if (world > 1 or args.loopback) else "none",
                    "l2": f"no flush: inputs ({32 * n_local / 1e9:.1f} GB of particles per GPU) >> 126 MB L2"},
         "per_gpu": value / world,
+        "step_ms_rank0": {"median": round(statistics.median(step_ms), 3), "min": round(min(step_ms), 3),
+                          "max": round(max(step_ms), 3)},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
                      "kernel": "k_advance (advance_p, one species per launch)",

@@ -136,6 +136,40 @@ def test_loopback_exchange_matches_periodic(V, field_solve, steps, device_exchan
         assert np.array_equal(fa, fb)       # static fields: halos move bytes only
 
 
+@pytest.mark.parametrize("walls", [False, True], ids=["periodic", "absorb_z"])
+@pytest.mark.parametrize("migration", ["rounds", "single"])
+@pytest.mark.parametrize("device_exchange", [False, True], ids=["nccl", "device"])
+def test_loopback_direct_kernel_matches_periodic(V, device_exchange, migration, walls):
+    """As above with the direct-load advance kernel (VPIC_OPT_ADVANCE_KERNEL =
+    1): its crossers leave through the same move_p / leave() code.  absorb_z:
+    absorbing z walls -- particles that enter the ghost layer through x/y and
+    then hit a wall there are removed exactly like in the local run."""
+    from paper_conf_sc_tanlta25_b200.pic import HotPath
+    g = inputs.GridSpec(7, 6, 5, dt=0.5, pbc=(0, 0, 2, 0, 0, 2) if walls else (0,) * 6)
+    wl = inputs.Workload("loopback_direct", g, [inputs.Species("electron", -1.0, 1.0, 0.7)], 30, 2, 0)
+    parts = inputs.make_species_particles(wl)
+    fields = inputs.make_fields(g, 0.05)
+    runs = []
+    for loop in (False, True):
+        hp = HotPath(wl, parts, fields, math=V.MATH_IEEE, loopback_exchange=loop, capacity_factor=1.0,
+                     device_exchange=loop and device_exchange, inbox_cap=4096,
+                     single_round=loop and migration == "single")
+        hp.ctx.set_option(V.VPIC_OPT_ADVANCE_KERNEL, 1)
+        for _ in range(2):
+            hp.step()
+        torch.cuda.synchronize()
+        runs.append(hp)
+    a, b = runs
+    pa, pb = a.particles_host(0), b.particles_host(0)
+    if walls:
+        assert pa.size < parts[0].size          # some were absorbed
+    assert np.array_equal(_multiset(pa), _multiset(pb))
+    assert not np.array_equal(pa.view(np.uint32), pb.view(np.uint32))
+    vox = g.interior_voxels()
+    ja, jb = a.jf.cpu().numpy()[vox], b.jf.cpu().numpy()[vox]
+    assert np.abs(ja - jb).max() <= 1e-5 * np.abs(ja).max() * 8
+
+
 @pytest.mark.parametrize("migration", ["rounds", "single"])
 def test_device_exchange_inbox_overflow_reported(V, migration):
     """An inbox smaller than one round's arrivals: the push keeps going,

@@ -48,6 +48,17 @@ def harris_small():
     return wh, inputs.make_species_particles(wh)
 
 
+def lpi_small():
+    """configs[4]'s laser-plasma slab (plasma in x in [nx/4, 3nx/4), hot
+    electrons u_th = 0.2 drifting at u_x = +0.3, cold heavy ions, static
+    laser ey = cbz = 0.02 sin(2 pi x / 32)) on a 64x8x8 grid, 24 ppc: the
+    high-crossing, empty-voxel case."""
+    from dataclasses import replace
+    wl = inputs.config(4)
+    wlp = replace(wl, grid=inputs.GridSpec(64, 8, 8), ppc=24)
+    return wlp, inputs.make_species_particles(wlp)
+
+
 # ------------------------------------------------------------------ sort --
 def sort_cases():
     out = []
@@ -134,6 +145,9 @@ def adv_cases():
     wh, ph = harris_small()
     out.append(("harris_sheet_electrons", wh.grid, ph[0], -1.0, 1.0,
                 inputs.make_fields(wh.grid, 0.01, kind="harris")))
+    wp, pp = lpi_small()
+    out.append(("lpi_slab_electrons", wp.grid, pp[0], -1.0, 1.0,
+                inputs.make_fields(wp.grid, 0.01, kind="lpi")))
     # random order on 40^3 voxels: every warp's items in distinct voxels
     gs = inputs.GridSpec(40, 40, 40)
     out.append(("scattered_cache_overflow", gs, inputs.random_particles(gs, 150000, 13, u_scale=0.5),

@@ -159,7 +159,7 @@ def run_oracle_steps(wl, n_steps, sort_every, order):
     oracle.build()
     g = wl.grid
     parts = inputs.make_species_particles(wl)
-    fields = inputs.make_fields(g, wl.field_amp)
+    fields = inputs.make_fields(g, wl.field_amp, kind=wl.kind)
     acc = np.zeros((g.nv, 12), np.float32)
     times = []
     pushes = 0
@@ -242,7 +242,7 @@ def our_arm(args, rank, world):
     parts = inputs.make_species_particles(wl, seed)
     if args.shuffle:
         parts = [inputs.shuffle(p, seed + 17 + k) for k, p in enumerate(parts)]
-    fields = inputs.make_fields(g, wl.field_amp, seed)
+    fields = inputs.make_fields(g, wl.field_amp, seed, kind=wl.kind)
     math_mode = vpic.MATH_IEEE if args.math == "ieee" else vpic.MATH_FAST
     dep = {"auto": 0, "lane": 1, "warp": 2}[args.deposit]
     cap = 1.0 if world == 1 else 1.05
@@ -369,7 +369,11 @@ def our_arm(args, rank, world):
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "f32",
-        "data": "synthetic (seeded Philox; uniform thermal e/ion plasma, quiet start)",
+        "data": "synthetic (seeded Philox; " + {
+            "uniform": "uniform thermal e/ion plasma, quiet start",
+            "harris": "Harris sheet: sech^2 density + background, tanh cB_x, drifting species, "
+                      "reflecting z",
+            "lpi": "laser-plasma slab: hot drifting electrons, cold ions, static laser ey = cbz"}[wl.kind] + ")",
         "config": {"workload": wl.name, "cells_per_gpu": [g.nx, g.ny, g.nz], "ppc_per_species": wl.ppc,
                    "species": len(wl.species), "particles": int(ntot), "sort_every": S,
                    "order": args.order, "shuffled": bool(args.shuffle), "math": args.math,

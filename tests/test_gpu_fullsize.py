@@ -29,7 +29,7 @@ def state(orc):
     wl = inputs.config(1)
     g = wl.grid
     parts = inputs.make_species_particles(wl)
-    fields = inputs.make_fields(g, wl.field_amp)
+    fields = inputs.make_fields(g, wl.field_amp, kind=wl.kind)
     hp = HotPath(wl, parts, fields, order=vpic.VPIC_SORT_STANDARD, math=vpic.MATH_FAST,
                  deposit=vpic.DEP_AUTO)
     hp.step(do_sort=True)      # sort (identity on the cell-major quiet start) + one PIC step
@@ -175,7 +175,7 @@ def test_fullsize_loopback_single_round_matches_local(device_exchange):
     wl = inputs.config(1)
     g = wl.grid
     parts = inputs.make_species_particles(wl)
-    fields = inputs.make_fields(g, wl.field_amp)
+    fields = inputs.make_fields(g, wl.field_amp, kind=wl.kind)
     out = []
     for loop in (False, True):
         hp = HotPath(wl, parts, fields, math=vpic.MATH_IEEE, loopback_exchange=loop,

@@ -144,13 +144,16 @@ def committed_traffic(kernel_key: str, workload: str):
 
 
 # --------------------------------------------------------- CPU / oracle --
-def oracle_sample_workload():
+def oracle_sample_workload(cfg: int = 1):
     """The reference arm's bounded sample: the same plasma recipe (species,
-    ppc, u_th, fields, sort period) on a 32x32x16 box."""
+    ppc, u_th, fields, boundaries, sort period) as configs[cfg] on a small box
+    (32x32x16 uniform; 32x16x32 Harris sheet; 64x16x16 LPI slab)."""
     from paper_conf_sc_tanlta25_b200 import inputs
     from dataclasses import replace
-    wl = inputs.config(1)
-    return replace(wl, grid=inputs.GridSpec(32, 32, 16), name=wl.name + "@32x32x16")
+    wl = inputs.config(3 if cfg == 3 else cfg)
+    n = {"uniform": (32, 32, 16), "harris": (32, 16, 32), "lpi": (64, 16, 16)}[wl.kind]
+    return replace(wl, grid=replace(wl.grid, nx=n[0], ny=n[1], nz=n[2]),
+                   name=wl.name + "@%dx%dx%d" % n)
 
 
 def run_oracle_steps(wl, n_steps, sort_every, order):
@@ -186,7 +189,7 @@ def inputs_config_name(args):
 def reference_arm(args, rank, world):
     if rank != 0:
         return
-    wl = oracle_sample_workload()
+    wl = oracle_sample_workload(args.config)
     S = args.sort_every or wl.sort_every
     order = ORDERS[args.order]
     _ = run_oracle_steps(wl, max(args.warmup, 0) and 1, S, order)  # untimed warm-up (1 step)
@@ -209,7 +212,7 @@ def reference_arm(args, rank, world):
 
 
 def cpu_baseline(args):
-    wl = oracle_sample_workload()
+    wl = oracle_sample_workload(args.config)
     S = args.sort_every or wl.sort_every
     times, per_step = run_oracle_steps(wl, 1, S, ORDERS[args.order])
     return {"value": per_step / times[0], "unit": UNIT, "cores": 1, "kind": "oracle",

@@ -47,6 +47,8 @@ import ctypes
 mb = ctypes.CDLL(os.path.join(ROOT, "tools", "mb_scatter.so"))
 P = lambda x: ctypes.c_void_p(x.data_ptr())
 print("mb gather ms", t(lambda: mb.mb_gather(P(src), P(out), P(perm), ctypes.c_int64(n))))
+for v, name in enumerate(["ldg", "nc.L2::64B", "nc.L1::no_allocate", "nc.L2::128B", "cg"]):
+    print("mb gather", name, "ms", t(lambda: mb.mb_gatherv(v, P(src), P(out), P(perm), ctypes.c_int64(n))))
 print("mb scatter ms", t(lambda: mb.mb_scatter(P(src), P(out), P(inv), ctypes.c_int64(n))))
 print("mb invert ms", t(lambda: mb.mb_invert(P(perm), P(inv), ctypes.c_int64(n))))
 print("ours (sort incl. gather) ms", t(lambda: vpic.vpic_sort_particles(hp.ctx, src, s.scratch, n, 0, 0, hp.ws)))

@@ -216,6 +216,15 @@ int vpic_advance_p(vpic_ctx *ctx, float q, float m, vpic_particle_t *p, int64_t 
                    const float *interp, float *acc, vpic_mover_t *movers, int64_t max_movers,
                    int64_t *n_movers, int32_t *flags, void *stream);
 
+/* Same, with the particle count in DEVICE memory (*np_dev, int64, 8-byte
+ * aligned; read by the kernels at run time, min(*np_dev, max_np) particles are
+ * pushed; max_np sizes the launch).  Lets a PIC step be captured in a CUDA
+ * graph and replayed while the count changes (with
+ * vpic_migrate_particles_dev).  Same argument rules otherwise. */
+int vpic_advance_p_dev(vpic_ctx *ctx, float q, float m, vpic_particle_t *p, const int64_t *np_dev,
+                       int64_t max_np, const float *interp, float *acc, vpic_mover_t *movers,
+                       int64_t max_movers, int64_t *n_movers, int32_t *flags, void *stream);
+
 /* ------------------------------------------------------ (a12) unload -- */
 
 /* jf on every edge of voxels 1..n+1 from the 4 accumulators sharing it,
@@ -293,6 +302,19 @@ int vpic_continuity_residual(vpic_ctx *ctx, const float *rho0, const float *rho1
 int vpic_migrate_particles(vpic_ctx *ctx, float q, float m, vpic_particle_t *p, int64_t *np,
                            int64_t max_np, vpic_mover_t *movers, const int64_t *n_movers,
                            float *acc, void *stream);
+
+/* vpic_migrate_particles with the count in DEVICE memory and no host
+ * synchronisation: every step is a stream operation, so it can be captured in
+ * a CUDA graph (a capture must hold an even number of calls: each call flips
+ * the inbox epoch, fixed at enqueue time).  Needs
+ * VPIC_OPT_SINGLE_ROUND_MIGRATION and VPIC_OPT_DEVICE_EXCHANGE (else
+ * VPIC_ERR_UNSUPPORTED).  *np_dev (int64) in/out; flags_dev (int32, device):
+ * capacity errors are OR-ed in as bits 1 (an inbox was full: particles lost),
+ * 2 (hole list full), 3 (arrivals did not fit max_np: dropped) -- check it
+ * when the count is read back.  n_movers is not reset. */
+int vpic_migrate_particles_dev(vpic_ctx *ctx, float q, float m, vpic_particle_t *p, int64_t *np_dev,
+                               int64_t max_np, const vpic_mover_t *movers, const int64_t *n_movers,
+                               float *acc, int32_t *flags_dev, void *stream);
 
 #ifdef __cplusplus
 }

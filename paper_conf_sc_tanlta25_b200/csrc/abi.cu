@@ -51,12 +51,12 @@ void note_launch(int n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
 cudaError_t launch_advance_p(const vpic_ctx *c, float qsp, float msp, vpic_particle_t *p,
                              int64_t np, const float *interp, float *acc, vpic_mover_t *movers,
                              int64_t max_movers, int64_t *n_movers, int32_t *flags,
-                             cudaStream_t s) {
+                             cudaStream_t s, const int64_t *np_dev) {
   if (c->math == MATH_IEEE)
     return launch_advance_p_ieee(c, qsp, msp, p, np, interp, acc, movers, max_movers, n_movers,
-                                 flags, s);
+                                 flags, s, np_dev);
   return launch_advance_p_fast(c, qsp, msp, p, np, interp, acc, movers, max_movers, n_movers,
-                               flags, s);
+                               flags, s, np_dev);
 }
 }  // namespace vpic
 
@@ -277,6 +277,22 @@ int vpic_advance_p(vpic_ctx *c, float q, float m, vpic_particle_t *p, int64_t np
                                       flags, S(stream)));
 }
 
+int vpic_advance_p_dev(vpic_ctx *c, float q, float m, vpic_particle_t *p, const int64_t *np_dev,
+                       int64_t max_np, const float *interp, float *acc, vpic_mover_t *movers,
+                       int64_t max_movers, int64_t *n_movers, int32_t *flags, void *stream) {
+  if (!c || !np_dev || max_np < 0 || max_np >= ((int64_t)1 << 31) || !(m > 0) || max_movers < 0)
+    return VPIC_ERR_INVALID;
+  if ((reinterpret_cast<uintptr_t>(np_dev) & 7u) != 0) return VPIC_ERR_INVALID;
+  if (max_np == 0) return VPIC_OK;
+  if (!p || !interp || !acc || !n_movers || !aligned16(p) || !aligned32(interp) || !aligned16(acc))
+    return VPIC_ERR_INVALID;
+  if (max_movers > 0 && (!movers || !aligned16(movers))) return VPIC_ERR_INVALID;
+  if ((reinterpret_cast<uintptr_t>(n_movers) & 7u) != 0) return VPIC_ERR_INVALID;
+  DeviceGuard dg(c->device);
+  return cuda_status(launch_advance_p(c, q, m, p, max_np, interp, acc, movers, max_movers, n_movers,
+                                      flags, S(stream), np_dev));
+}
+
 int vpic_unload_accumulator(vpic_ctx *c, const float *acc, float *jf, void *stream) {
   if (!c || !acc || !jf || !aligned16(acc) || !aligned16(jf)) return VPIC_ERR_INVALID;
   DeviceGuard dg(c->device);
@@ -342,6 +358,17 @@ int vpic_migrate_particles(vpic_ctx *c, float q, float m, vpic_particle_t *p, in
   if (*np > 0 && (!p || !aligned16(p))) return VPIC_ERR_INVALID;
   DeviceGuard dg(c->device);
   return migrate(c, q, m, p, np, max_np, movers, n_movers, acc, S(stream));
+}
+
+int vpic_migrate_particles_dev(vpic_ctx *c, float q, float m, vpic_particle_t *p, int64_t *np_dev,
+                               int64_t max_np, const vpic_mover_t *movers, const int64_t *n_movers,
+                               float *acc, int32_t *flags_dev, void *stream) {
+  (void)q; (void)m;
+  if (!c || !np_dev || max_np < 0 || max_np >= ((int64_t)1 << 31) || !n_movers || !acc || !p ||
+      !aligned16(p) || !flags_dev)
+    return VPIC_ERR_INVALID;
+  DeviceGuard dg(c->device);
+  return migrate_dev(c, p, np_dev, max_np, movers, n_movers, acc, flags_dev, S(stream));
 }
 
 }  // extern "C"

@@ -225,6 +225,19 @@ __global__ void k_lsa_barrier(ncclDevComm dc) {
 }
 
 __global__ void k_di_set(int64_t *ctr, int64_t np) { ctr[0] = np; ctr[3] = 0; }
+__global__ void k_di_set_dev(int64_t *ctr, const int64_t *np_dev) { ctr[0] = *np_dev; ctr[3] = 0; }
+// device-count call done: the new count out; the capacity flags (di_flag bit
+// 0 inbox full, 1 hole list full, 2 arrivals did not fit; dflag) OR-ed into
+// the caller's flags shifted up by one (bit 0 stays advance_p's mover
+// overflow) and cleared for the next call
+__global__ void k_di_finish(const int64_t *ctr, int64_t *np_dev, int32_t *dflag, int32_t *di_flag,
+                            int32_t *flags_dev) {
+  *np_dev = ctr[0];
+  const int32_t f = *dflag | *di_flag;
+  if (f) *flags_dev |= (f << 1);
+  *dflag = 0;
+  *di_flag = 0;
+}
 
 // Holes of this round: H = departures in `mv` (device count *hdev).
 __global__ void k_di_holes_prep(int64_t *ctr, const int64_t *hdev, int64_t hcap, int32_t *flag) {
@@ -799,6 +812,32 @@ int migrate_ghost_di(vpic_ctx *c, vpic_particle_t *p, int64_t *np_io, int64_t ma
 }
 
 }  // namespace
+
+// The same with the particle count on the device and no host
+// synchronisation: every step is a stream operation (kernels, memsets, NCCL
+// plane send/recv), so a PIC step or a whole sort period can be captured in a
+// CUDA graph and replayed.  The epoch parity is fixed at enqueue time (each
+// call flips it), so a captured sequence must hold an even number of calls.
+int migrate_dev(vpic_ctx *c, vpic_particle_t *p, int64_t *np_dev, int64_t max_np,
+                const vpic_mover_t *movers, const int64_t *n_movers, float *acc, int32_t *flags_dev,
+                cudaStream_t s) {
+  Exchange *ex = c->ex;
+  if (!ex || !ex->di || !c->gk.ghost_mig) return VPIC_ERR_UNSUPPORTED;
+  const int e = (int)(c->di_epoch & 1);
+  int32_t *d_flags = reinterpret_cast<int32_t *>(c->d_count + 1);
+  CKC(cudaMemsetAsync(d_flags, 0, 4, s));
+  k_di_set_dev<<<1, 1, 0, s>>>(ex->di_ctr, np_dev); note_launch();
+  if (int rc = di_remove_holes(c, p, movers, n_movers, s)) return rc;
+  unsigned char *inbox = static_cast<unsigned char *>(ex->di_buf);
+  k_lsa_barrier<<<1, 128, 0, s>>>(ex->di_dcomm); note_launch();
+  k_di_take_ghost<<<1, 32, 0, s>>>(inbox, e, ex->di_cap, max_np, ex->di_ctr, ex->di_flag); note_launch();
+  k_di_unpack_ghost<<<(unsigned)c->num_sms * 4, 256, 0, s>>>(inbox, e, ex->di_cap, ex->di_ctr, p); note_launch();
+  CKC(cudaGetLastError());
+  c->di_epoch++;
+  if (int rc = reduce_acc_ghosts(c, acc, s)) return rc;
+  k_di_finish<<<1, 1, 0, s>>>(ex->di_ctr, np_dev, d_flags, ex->di_flag, flags_dev); note_launch();
+  return cudaGetLastError() == cudaSuccess ? VPIC_OK : VPIC_ERR_CUDA;
+}
 
 // Up to 3 rounds: pack movers per face, exchange counts, exchange records,
 // remove departed / absorbed particles, append arrivals, continue their move.

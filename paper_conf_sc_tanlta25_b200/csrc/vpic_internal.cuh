@@ -107,19 +107,21 @@ namespace vpic {
 void note_launch(int n = 1);
 
 // ---- launchers implemented in the .cu files (return cudaError_t) ----------
+// np_dev (nullable): the live count is read on the device (min(*np_dev, np));
+// np then only bounds it and sizes the launch
 cudaError_t launch_advance_p(const vpic_ctx *c, float qsp, float msp, vpic_particle_t *p,
                              int64_t np, const float *interp, float *acc, vpic_mover_t *movers,
                              int64_t max_movers, int64_t *n_movers, int32_t *flags,
-                             cudaStream_t s);
+                             cudaStream_t s, const int64_t *np_dev = nullptr);
 // the two math variants are compiled from the same source (advance_p.cu)
 cudaError_t launch_advance_p_fast(const vpic_ctx *c, float qsp, float msp, vpic_particle_t *p,
                                   int64_t np, const float *interp, float *acc,
                                   vpic_mover_t *movers, int64_t max_movers, int64_t *n_movers,
-                                  int32_t *flags, cudaStream_t s);
+                                  int32_t *flags, cudaStream_t s, const int64_t *np_dev = nullptr);
 cudaError_t launch_advance_p_ieee(const vpic_ctx *c, float qsp, float msp, vpic_particle_t *p,
                                   int64_t np, const float *interp, float *acc,
                                   vpic_mover_t *movers, int64_t max_movers, int64_t *n_movers,
-                                  int32_t *flags, cudaStream_t s);
+                                  int32_t *flags, cudaStream_t s, const int64_t *np_dev = nullptr);
 // move_p of a list of movers (incoming particles after migration)
 // n_in_dev (nullable): device count, n_in then only bounds it; di_round: the
 // migration round of the departures (device-initiated exchange only)
@@ -159,6 +161,11 @@ cudaError_t launch_sort(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_
 
 int migrate(vpic_ctx *c, float qsp, float msp, vpic_particle_t *p, int64_t *np, int64_t max_np,
             vpic_mover_t *movers, const int64_t *n_movers, float *acc, cudaStream_t s);
+// single-round, device-initiated migration with the particle count on the
+// device: no host synchronisation (capturable in a CUDA graph)
+int migrate_dev(vpic_ctx *c, vpic_particle_t *p, int64_t *np_dev, int64_t max_np,
+                const vpic_mover_t *movers, const int64_t *n_movers, float *acc, int32_t *flags_dev,
+                cudaStream_t s);
 int exchange_create(vpic_ctx *c, const uint8_t *uid);
 void exchange_destroy(vpic_ctx *c);
 // dir = +1: fill the +x/+y/+z ghost planes from the +neighbours' plane 1;

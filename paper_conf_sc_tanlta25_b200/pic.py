@@ -31,6 +31,7 @@ class SpeciesState:
     movers: torch.Tensor     # [max_movers, 4]
     n_movers: torch.Tensor   # int64[1]
     flags: torch.Tensor      # int32[1]
+    np_dev: torch.Tensor = None   # int64[1]: the count on the device (graph mode)
 
 
 class HotPath:
@@ -40,7 +41,8 @@ class HotPath:
                  uid: bytes = None, capacity_factor: float = 1.0, max_movers: int = 1 << 20,
                  device: Optional[int] = None, field_solve: bool = False, eps0: float = 1.0,
                  loopback_exchange: bool = False, concurrent_species: bool = False,
-                 device_exchange: bool = False, inbox_cap: int = 0, single_round: bool = False):
+                 device_exchange: bool = False, inbox_cap: int = 0, single_round: bool = False,
+                 graphs: bool = False):
         vpic.load()
         self.wl = wl
         self.g = wl.grid
@@ -90,6 +92,21 @@ class HotPath:
             max_np = max(max_np, cap)
         ws = vpic.vpic_sort_workspace_bytes(self.ctx, max_np, order)
         self.ws = torch.empty(max(ws, 1), dtype=torch.uint8, device=self.dev)
+        # CUDA-graph mode: the PIC steps of a sort period are captured once per
+        # particle-buffer configuration and replayed; particle counts live on
+        # the device (vpic_advance_p_dev / vpic_migrate_particles_dev: no host
+        # synchronisation inside a period).  Needs no migration, or the
+        # single-round device-initiated exchange.
+        self.graphs = graphs
+        if graphs:
+            if self.migrate and not (single_round and device_exchange):
+                raise ValueError("graphs need the single-round device-initiated exchange (or none)")
+            if self.concurrent:
+                raise ValueError("graphs and concurrent species are exclusive")
+            for sp in self.species:
+                sp.np_dev = torch.tensor([sp.np], dtype=torch.int64, device=self.dev)
+        self._graphs = {}
+        self._warm = False
         self.adv_events = []   # (start, end) CUDA events around advance_p, when recording
         self.sort_events = []  # (start, end, species) around vpic_sort_particles
         self.record_advance = False
@@ -156,8 +173,64 @@ class HotPath:
 
     def cycle(self, steps: int):
         """One sort period: sort, then `steps` PIC steps."""
+        if self.graphs:
+            return self._cycle_graph(steps)
         for k in range(steps):
             self.step(do_sort=(k == 0))
+
+    # ------------------------------------------------------- graph mode --
+    def sync_counts(self):
+        """Graph mode: bring the device particle counts (and capacity flags)
+        back to the host."""
+        if not self.graphs:
+            return
+        torch.cuda.current_stream().synchronize()
+        for s in self.species:
+            s.np = int(s.np_dev.item())
+            fl = int(s.flags.item())
+            if fl:
+                raise vpic.VpicError(f"graph-mode step ({s.name}: flags {fl:#x})", vpic.VPIC_ERR_CAPACITY)
+
+    def _step_dev(self):
+        vpic.vpic_load_interpolator(self.ctx, self.fields, self.interp)
+        vpic.vpic_clear_accumulator(self.ctx, self.acc)
+        for s in self.species:
+            vpic.vpic_advance_p_dev(self.ctx, s.q, s.m, s.p, s.np_dev, s.p.shape[0], self.interp, self.acc,
+                                    s.movers, s.movers.shape[0], s.n_movers, s.flags)
+            if self.migrate:
+                vpic.vpic_migrate_particles_dev(self.ctx, s.q, s.m, s.p, s.np_dev, s.p.shape[0], s.movers,
+                                                s.n_movers, self.acc, s.flags)
+                s.n_movers.zero_()
+        vpic.vpic_unload_accumulator(self.ctx, self.acc, self.jf)
+        if self.field_solve:
+            vpic.vpic_advance_b(self.ctx, self.fields, 0.5)
+            vpic.vpic_advance_e(self.ctx, self.fields, self.jf, self.eps0)
+            vpic.vpic_advance_b(self.ctx, self.fields, 0.5)
+
+    def _cycle_graph(self, steps: int):
+        self.sync_counts()
+        self.sort()
+        for s in self.species:
+            s.np_dev.fill_(s.np)
+        if self.migrate and (steps * len(self.species)) % 2:
+            for _ in range(steps):     # (an odd number of exchanges cannot be replayed)
+                self._step_dev()
+            return
+        key = (steps, tuple(s.p.data_ptr() for s in self.species), self.fields.data_ptr())
+        if not self._warm:             # first period eagerly: lazy allocations, attributes
+            for _ in range(steps):
+                self._step_dev()
+            self._warm = True
+            return
+        gr = self._graphs.get(key)
+        if gr is None:
+            torch.cuda.synchronize()
+            gr = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(gr):
+                for _ in range(steps):
+                    self._step_dev()
+            self._graphs[key] = gr
+        gr.replay()
 
     # ------------------------------------------------------- host <-> device --
     def run_host_cycles(self, host_in, host_out, fields_host, jf_host, n_cycles: int, S: int):
@@ -235,8 +308,11 @@ class HotPath:
         return pushes
 
     def particles_host(self, k: int) -> np.ndarray:
+        self.sync_counts()
         s = self.species[k]
         return vpic.particles_to_host(s.p[:s.np])
 
     def close(self):
+        torch.cuda.synchronize()
+        self._graphs.clear()        # captured graphs reference the context's NCCL state
         self.ctx.close()

@@ -184,3 +184,42 @@ def test_device_exchange_inbox_overflow_reported(V, migration):
     with pytest.raises(V.VpicError) as ei:
         hp.step()
     assert ei.value.status == -2      # VPIC_ERR_CAPACITY
+
+
+@pytest.mark.timeout(300)
+@pytest.mark.parametrize("exchange", ["none", "loopback"])
+def test_graph_mode_matches_eager(V, exchange):
+    """HotPath(graphs=True): the PIC steps of each sort period captured once per
+    particle-buffer configuration (CUDA graph) and replayed, particle counts on
+    the device (vpic_advance_p_dev / vpic_migrate_particles_dev).  Three sort
+    periods (eager warm-up, capture + replay, replay of the other buffer
+    configuration's graph...) must reproduce the eager run: bit-identical
+    arrays without exchange, equal multisets with the loopback single-round
+    exchange; jf within the reordering tolerance."""
+    import gc
+    from paper_conf_sc_tanlta25_b200.pic import HotPath
+    gc.collect()                        # no other test's context (NCCL communicator) alive
+    g = inputs.GridSpec(8, 6, 5, dt=0.5)
+    wl = inputs.Workload("graphs", g, [inputs.Species("electron", -1.0, 1.0, 0.6),
+                                       inputs.Species("ion", 1.0, 4.0, 0.3)], 40, 4, 4)
+    parts = inputs.make_species_particles(wl)
+    fields = inputs.make_fields(g, 0.05)
+    loop = exchange == "loopback"
+    res = []
+    for graphs in (False, True):      # one context (one NCCL communicator) at a time
+        hp = HotPath(wl, parts, fields, math=V.MATH_IEEE, loopback_exchange=loop, device_exchange=loop,
+                     single_round=loop, inbox_cap=4096, capacity_factor=1.0, graphs=graphs)
+        for _ in range(4):
+            hp.cycle(4)
+        torch.cuda.synchronize()
+        res.append(([hp.particles_host(k) for k in range(2)], hp.jf.cpu().numpy(), len(hp._graphs)))
+        hp.close()
+    (pa, ja, _), (pb, jb, ng) = res
+    assert ng == 2                      # one graph per buffer configuration, replayed
+    for k in range(2):
+        if loop:
+            assert np.array_equal(_multiset(pa[k]), _multiset(pb[k]))
+        else:
+            assert np.array_equal(pa[k].view(np.uint32), pb[k].view(np.uint32))
+    vox = g.interior_voxels()
+    assert np.abs(ja[vox] - jb[vox]).max() <= 1e-5 * np.abs(ja[vox]).max() * 8

@@ -33,7 +33,7 @@ DEP_AUTO, DEP_LANE, DEP_WARP = 0, 1, 2
 EXPORTS = ["vpic_get_unique_id", "vpic_ctx_create", "vpic_ctx_destroy", "vpic_ctx_set_option",
            "vpic_ctx_info", "vpic_status_string", "vpic_sort_workspace_bytes",
            "vpic_sort_particles", "vpic_load_interpolator", "vpic_clear_accumulator",
-           "vpic_advance_p", "vpic_unload_accumulator", "vpic_migrate_particles",
+           "vpic_advance_p", "vpic_advance_p_dev", "vpic_unload_accumulator", "vpic_migrate_particles", "vpic_migrate_particles_dev",
            "vpic_kernel_launches", "vpic_advance_b", "vpic_advance_e", "vpic_gather_scatter",
            "vpic_accumulate_rho", "vpic_continuity_residual"]
 

@@ -47,7 +47,7 @@ def parse():
     ap.add_argument("--shuffle", action="store_true", help="random initial order (paper's 'random')")
     ap.add_argument("--sort-every", type=int, default=0)
     ap.add_argument("--math", default="fast", choices=["fast", "ieee"])
-    ap.add_argument("--deposit", default="auto", choices=["auto", "lane", "warp", "cache"])
+    ap.add_argument("--deposit", default="auto", choices=["auto", "lane", "warp"])
     ap.add_argument("--kernel", default="auto", choices=["auto", "direct", "tma"])
     ap.add_argument("--field-solve", action="store_true",
                     help="full PIC step: + advance_b/advance_e (self-consistent fields)")
@@ -247,7 +247,7 @@ def our_arm(args, rank, world):
         parts = [inputs.shuffle(p, seed + 17 + k) for k, p in enumerate(parts)]
     fields = inputs.make_fields(g, wl.field_amp, seed, kind=wl.kind)
     math_mode = vpic.MATH_IEEE if args.math == "ieee" else vpic.MATH_FAST
-    dep = {"auto": 0, "lane": 1, "warp": 2, "cache": 3}[args.deposit]
+    dep = {"auto": 0, "lane": 1, "warp": 2}[args.deposit]
     cap = 1.0 if world == 1 else 1.05
     hp = HotPath(wl, parts, fields, order=order, math=math_mode, deposit=dep, rank=rank,
                  nranks=world, uid=uid, capacity_factor=cap, device=local,

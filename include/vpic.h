@@ -72,12 +72,7 @@ enum {
   VPIC_OPT_MATH = 0,
   /* current scatter strategy: 0 = AUTO, 1 = LANE (3 x red.global.add.v4.f32 per
    * streak), 2 = WARP (same-voxel contributions reduced across the warp with
-   * shuffles before red.global; falls back to LANE for scattered warps),
-   * 3 = CACHE (WARP, plus a warp-private shared-memory cache of accumulator
-   * rows over a 4x4x3 voxel window: scattered in-cell streaks are summed in
-   * shared memory and reach acc when their row is evicted or at kernel end;
-   * each warp pushes one contiguous range of the particle array; TMA kernel
-   * only, the direct kernel treats it as WARP).
+   * shuffles before red.global; falls back to LANE for scattered warps).
    * Default AUTO (= WARP). */
   VPIC_OPT_DEPOSIT = 1,
   /* default TileSz for VPIC_SORT_TILED_STRIDED when tile_sz == 0.  Default

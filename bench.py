@@ -230,10 +230,17 @@ def our_arm(args, rank, world):
     local = int(os.environ.get("LOCAL_RANK", "0"))
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    wl = inputs.config(3 if world > 1 else args.config)
+    # N > 1: weak scaling on configs[3] (C2 per GPU), or strong scaling of
+    # the LPI slab (configs[4], --config 4: the 512x256x256 box split over
+    # the process grid)
+    strong = world > 1 and args.config == 4
+    wl = inputs.config(args.config if (world == 1 or strong) else 3)
     S = args.sort_every or wl.sort_every
     order = ORDERS[args.order]
-    g = inputs.decompose(wl.grid, world, rank) if world > 1 else wl.grid
+    if strong:
+        g = inputs.strong_decompose(wl.grid, world, rank)
+    else:
+        g = inputs.decompose(wl.grid, world, rank) if world > 1 else wl.grid
     from dataclasses import replace
     wl = replace(wl, grid=g)
     uid = None
@@ -248,9 +255,17 @@ def our_arm(args, rank, world):
     fields = inputs.make_fields(g, wl.field_amp, seed, kind=wl.kind)
     math_mode = vpic.MATH_IEEE if args.math == "ieee" else vpic.MATH_FAST
     dep = {"auto": 0, "lane": 1, "warp": 2}[args.deposit]
-    cap = 1.0 if world == 1 else 1.05
+    # particle capacity per rank: the drifting LPI electrons pile up on the
+    # downstream ranks (~0.13% of a rank's electrons cross each step at 2
+    # GPUs); movers per inbox slot: a boundary plane's electrons x 0.35 (the
+    # crossing fraction per step of a drift-0.3, u_th-0.2 population is ~0.17)
+    cap = 1.0 if world == 1 else (1.5 if strong else 1.05)
+    inbox = 0
+    if strong:
+        plane = max(g.ny * g.nz, g.nx * g.nz, g.nx * g.ny)
+        inbox = max(1 << 19, int(0.35 * wl.ppc * plane))
     hp = HotPath(wl, parts, fields, order=order, math=math_mode, deposit=dep, rank=rank,
-                 nranks=world, uid=uid, capacity_factor=cap, device=local,
+                 nranks=world, uid=uid, capacity_factor=cap, device=local, inbox_cap=inbox,
                  field_solve=args.field_solve, loopback_exchange=args.loopback and world == 1,
                  concurrent_species=args.concurrent_species,
                  device_exchange=args.exchange in ("auto", "device") and (world > 1 or args.loopback),
@@ -371,13 +386,16 @@ def our_arm(args, rank, world):
     out = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+        "scaling": "strong" if strong else "weak", "vs_baseline": None, "dtype": "f32",
         "data": "synthetic (seeded Philox; " + {
             "uniform": "uniform thermal e/ion plasma, quiet start",
             "harris": "Harris sheet: sech^2 density + background, tanh cB_x, drifting species, "
                       "reflecting z",
             "lpi": "laser-plasma slab: hot drifting electrons, cold ions, static laser ey = cbz"}[wl.kind] + ")",
-        "config": {"workload": wl.name, "cells_per_gpu": [g.nx, g.ny, g.nz], "ppc_per_species": wl.ppc,
+        "config": {"workload": wl.name, "cells_per_gpu": [g.nx, g.ny, g.nz],
+                   "global_cells": ([g.gnx or g.nx, g.ny * inputs.process_grid(world)[1],
+                                     g.nz * inputs.process_grid(world)[2]] if strong else None),
+                   "ppc_per_species": wl.ppc,
                    "species": len(wl.species), "particles": int(ntot), "sort_every": S,
                    "order": args.order, "shuffled": bool(args.shuffle), "math": args.math,
                    "deposit": args.deposit, "kernel": args.kernel,

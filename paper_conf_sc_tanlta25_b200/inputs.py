@@ -51,6 +51,7 @@ class GridSpec:
     gx0: int = 0
     gy0: int = 0
     gz0: int = 0
+    gnx: int = 0        # global box width along x (0: this block is the whole box)
 
     @property
     def nv(self) -> int:
@@ -199,10 +200,14 @@ def harris_cells(g: GridSpec, ppc_mean: int, seed: int, sp_index: int) -> np.nda
 
 
 def lpi_cells(g: GridSpec, ppc: int) -> np.ndarray:
-    """Plasma slab x in [nx/4, 3nx/4), ppc per slab cell."""
-    x0, x1 = g.nx // 4, 3 * g.nx // 4
+    """Plasma slab x in [G/4, 3G/4) of the global box (G = g.gnx, or g.nx
+    for an undecomposed box), ppc per slab cell: this block's part of it
+    (global cell gx0 + x - 1 is local interior column x)."""
+    G = g.gnx or g.nx
+    x0 = max(G // 4 - g.gx0, 0)
+    x1 = min(3 * G // 4 - g.gx0, g.nx)
     z, y, x = np.meshgrid(np.arange(1, g.nz + 1), np.arange(1, g.ny + 1),
-                          np.arange(x0 + 1, x1 + 1), indexing="ij")
+                          np.arange(x0 + 1, max(x1, x0) + 1), indexing="ij")
     return np.repeat(g.voxel(x, y, z).reshape(-1).astype(np.int32), ppc)
 
 
@@ -293,3 +298,16 @@ def decompose(block: GridSpec, nranks: int, rank: int) -> GridSpec:
     n = (block.nx, block.ny, block.nz)
     return replace(block, nbr_rank=tuple(nbr), rank=rank,
                    gx0=c[0] * n[0], gy0=c[1] * n[1], gz0=c[2] * n[2])
+
+
+def strong_decompose(box: GridSpec, nranks: int, rank: int) -> GridSpec:
+    """Rank `rank`'s block when the periodic box `box` is SPLIT over the
+    process grid of `nranks` (strong scaling: fixed global size, configs[4]);
+    every dimension must divide."""
+    P = process_grid(nranks)
+    n = (box.nx, box.ny, box.nz)
+    if any(n[a] % P[a] for a in range(3)):
+        raise ValueError(f"{n} cells do not split over the process grid {P}")
+    block = replace(box, nx=box.nx // P[0], ny=box.ny // P[1], nz=box.nz // P[2],
+                    gnx=box.gnx or box.nx)
+    return decompose(block, nranks, rank)

@@ -255,6 +255,36 @@ def test_decompose_neighbours():
                 assert g.nbr_rank == (0,) * 6
 
 
+
+def test_strong_decompose_lpi_slab():
+    """Strong scaling of configs[4] (bench.py --config 4 at N > 1): the box is
+    split over the process grid, and the ranks' slab cells and laser fields
+    reassemble exactly the undecomposed box's (slab x in [G/4, 3G/4))."""
+    box = inputs.GridSpec(32, 8, 8)
+    ref = set()
+    for v in inputs.lpi_cells(box, 1):
+        x, y, z = box.coords(v)
+        ref.add((int(x), int(y), int(z)))
+    fref = inputs.make_fields(box, 0.0, kind="lpi")
+    for n in (2, 4, 8):
+        got = []
+        for r in range(n):
+            g = inputs.strong_decompose(box, n, r)
+            assert (g.gnx, g.nx * inputs.process_grid(n)[0]) == (32, 32)
+            for v in inputs.lpi_cells(g, 1):
+                x, y, z = g.coords(v)
+                assert 1 <= x <= g.nx
+                got.append((int(x) + g.gx0, int(y) + g.gy0, int(z) + g.gz0))
+            # laser phase follows the global x of every interior voxel
+            f = inputs.make_fields(g, 0.0, kind="lpi")
+            for v in g.interior_voxels()[:: max(1, g.ncells // 50)]:
+                x, y, z = g.coords(v)
+                gv = box.voxel(x + g.gx0, y + g.gy0, z + g.gz0)
+                assert f[v, 1] == fref[gv, 1] and f[v, 6] == fref[gv, 6]
+        assert len(got) == len(set(got)) and set(got) == ref, n
+    with pytest.raises(ValueError):
+        inputs.strong_decompose(inputs.GridSpec(5, 4, 4), 2, 0)
+
 # ------------------------------------------------ single-round migration --
 # Host logic of VPIC_OPT_SINGLE_ROUND_MIGRATION (csrc/migrate.cu:
 # ghost_migration_enable, migrate_ghost, reduce_acc_ghosts), replayed with

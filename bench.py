@@ -181,15 +181,18 @@ def run_oracle_steps(wl, n_steps, sort_every, order):
     return times, sum(p.size for p in parts) * sort_every
 
 
-def inputs_config_name(args):
-    from paper_conf_sc_tanlta25_b200 import inputs
-    return inputs.config(args.config).name
+def effective_config(args, world):
+    """The configs[] index a run measures: as given on one GPU; under torchrun
+    the weak-scaling configs[3], or configs[4] split over the ranks (strong)."""
+    return args.config if (world == 1 or args.config == 4) else 3
 
 
 def reference_arm(args, rank, world):
     if rank != 0:
         return
-    wl = oracle_sample_workload(args.config)
+    from paper_conf_sc_tanlta25_b200 import inputs
+    cfg = effective_config(args, world)
+    wl = oracle_sample_workload(cfg)
     S = args.sort_every or wl.sort_every
     order = ORDERS[args.order]
     _ = run_oracle_steps(wl, max(args.warmup, 0) and 1, S, order)  # untimed warm-up (1 step)
@@ -199,9 +202,10 @@ def reference_arm(args, rank, world):
     out = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * total / args.steps,
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+        "higher_is_better": True, "scaling": "strong" if (world > 1 and cfg == 4) else "weak",
+        "vs_baseline": None, "dtype": "f32",
         "data": "synthetic",
-        "config": {"workload": inputs_config_name(args), "order": args.order, "sort_every": S,
+        "config": {"workload": inputs.config(cfg).name, "order": args.order, "sort_every": S,
                    "sample": f"{wl.name}: {per_step // S} particles per step (bounded CPU sample)"},
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
                          "sample": f"serial C++ oracle (oracle/), {wl.name}: {per_step // S} particles, "
@@ -234,7 +238,7 @@ def our_arm(args, rank, world):
     # the LPI slab (configs[4], --config 4: the 512x256x256 box split over
     # the process grid)
     strong = world > 1 and args.config == 4
-    wl = inputs.config(args.config if (world == 1 or strong) else 3)
+    wl = inputs.config(effective_config(args, world))
     S = args.sort_every or wl.sort_every
     order = ORDERS[args.order]
     if strong:

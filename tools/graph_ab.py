@@ -15,13 +15,16 @@ from paper_conf_sc_tanlta25_b200.pic import HotPath
 ap = argparse.ArgumentParser()
 ap.add_argument("--periods", type=int, default=3)
 ap.add_argument("--config", type=int, default=1)
+ap.add_argument("--loopback", action="store_true",
+                help="every periodic face through the single-round device-initiated exchange")
 a = ap.parse_args()
 wl = inputs.config(a.config)
 parts = inputs.make_species_particles(wl, inputs.MASTER_SEED + 1)
 fields = inputs.make_fields(wl.grid, wl.field_amp, inputs.MASTER_SEED + 1, kind=wl.kind)
 S = wl.sort_every
 for graphs in (False, True, False, True):
-    hp = HotPath(wl, parts, fields, graphs=graphs)
+    kw = dict(loopback_exchange=True, device_exchange=True, single_round=True) if a.loopback else {}
+    hp = HotPath(wl, parts, fields, graphs=graphs, **kw)
     for _ in range(2):
         hp.cycle(S)
     torch.cuda.synchronize()
@@ -32,7 +35,8 @@ for graphs in (False, True, False, True):
     e1.record()
     torch.cuda.synchronize()
     ms = e0.elapsed_time(e1) / a.periods
-    print(f"graphs={graphs} {ms:.2f} ms per period, {S * hp.n_particles / ms / 1e6:.2f} G pushes/s", flush=True)
+    hp.sync_counts()
+    print(f"loopback={a.loopback} graphs={graphs} {ms:.2f} ms per period, {S * hp.n_particles / ms / 1e6:.2f} G pushes/s", flush=True)
     hp.close()
     del hp
     torch.cuda.empty_cache()

@@ -511,11 +511,10 @@ cudaError_t radix_pass_bits(const uint32_t *kin, const uint32_t *vin, uint32_t *
                             unsigned long long *status, unsigned int *ctr, cudaStream_t s) {
   const size_t smem = (size_t)NW * (1 << BITS) * 2 + (size_t)(1 << BITS) * 8 + (size_t)TILE * 8;
   const int64_t tiles = (n + TILE - 1) / TILE;
-  static bool configured = false;
-  if (!configured) {   // > 48 KB only for large tiles; set once per instantiation
+  static std::atomic<uint64_t> configured{0};   // > 48 KB only for large tiles; once per device
+  once_per_device(configured, [&] {
     cudaFuncSetAttribute(k_radix_pass<BITS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    configured = true;
-  }
+  });
   k_radix_pass<BITS><<<(unsigned)tiles, NT, smem, s>>>(kin, vin, kout, vout, n, shift, dig_off,
                                                        status, ctr); note_launch();
   return cudaGetLastError();
@@ -658,11 +657,10 @@ cudaError_t launch_sort(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_
     {
       int tot = 0;
       for (int q = 0; q < pr.npass; ++q) tot += 1 << pr.bits[q];
-      static bool configured = false;
-      if (!configured) {
+      static std::atomic<uint64_t> configured{0};
+      once_per_device(configured, [] {
         cudaFuncSetAttribute(k_rank_keys, cudaFuncAttributeMaxDynamicSharedMemorySize, 4 * MAX_PASSES * (1 << MAX_BITS));
-        configured = true;
-      }
+      });
       k_rank_keys<<<grid_cap(np, 256, sms, 2), 256, 4 * (size_t)tot, s>>>(
           K, P, offs, np, order, T, max_r, ck, pr, ghist, new_keys); note_launch();
       CK(cudaGetLastError());

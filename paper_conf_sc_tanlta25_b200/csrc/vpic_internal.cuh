@@ -5,6 +5,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <atomic>
+
 #include "../../include/vpic.h"
 
 namespace vpic {
@@ -105,6 +107,23 @@ namespace vpic {
 
 // process-wide count of kernels launched by the library (vpic_kernel_launches)
 void note_launch(int n = 1);
+
+// Run f() (e.g. cudaFuncSetAttribute, a per-device setting) once per device
+// for the current device; `done` is the caller's static bitmask of devices.
+// Concurrent first calls may both run f() (idempotent); nobody launches
+// before it has completed on its device.
+template <class F>
+inline void once_per_device(std::atomic<uint64_t> &done, F &&f) {
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) {
+    f();
+    return;
+  }
+  const uint64_t bit = 1ull << dev;
+  if (done.load(std::memory_order_acquire) & bit) return;
+  f();
+  done.fetch_or(bit, std::memory_order_release);
+}
 
 // ---- launchers implemented in the .cu files (return cudaError_t) ----------
 // np_dev (nullable): the live count is read on the device (min(*np_dev, np));

@@ -231,9 +231,12 @@ def our_arm(args, rank, world):
     from paper_conf_sc_tanlta25_b200 import inputs, vpic
     from paper_conf_sc_tanlta25_b200.pic import HotPath
 
+    from paper_conf_sc_tanlta25_b200.pic import bind_to_gpu_cpus
     local = int(os.environ.get("LOCAL_RANK", "0"))
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
+    # pinned e2e buffers first-touched on the GPU's NUMA node (2-socket nodes)
+    cpu_bind = bind_to_gpu_cpus(local)
     # N > 1: weak scaling on configs[3] (C2 per GPU), or strong scaling of
     # the LPI slab (configs[4], --config 4: the 512x256x256 box split over
     # the process grid)
@@ -409,6 +412,7 @@ def our_arm(args, rank, world):
                                if (world > 1 or args.loopback) else "none",
                    "migration": ("rounds" if args.migration == "rounds" else "single")
                                 if (world > 1 or args.loopback) else "none",
+                   "cpu_bind": cpu_bind,
                    "l2": f"no flush: inputs ({32 * n_local / 1e9:.1f} GB of particles per GPU) >> 126 MB L2"},
         "per_gpu": value / world,
         "step_ms_rank0": {"median": round(statistics.median(step_ms), 3), "min": round(min(step_ms), 3),

@@ -20,6 +20,33 @@ import torch
 from . import inputs, vpic
 
 
+def bind_to_gpu_cpus(device: int) -> Optional[int]:
+    """Restrict this process to the CPUs NVML reports as local to `device`
+    (its NUMA node), so pinned host buffers allocated afterwards are
+    first-touched next to the GPU's PCIe root. Returns the number of CPUs
+    bound to, or None when NVML cannot tell (nothing changed)."""
+    import os
+    try:
+        import pynvml
+        p = torch.cuda.get_device_properties(device)
+        bus = "%08x:%02x:%02x.0" % (p.pci_domain_id, p.pci_bus_id, p.pci_device_id)
+        pynvml.nvmlInit()
+        try:
+            h = pynvml.nvmlDeviceGetHandleByPciBusId(bus)
+            ncpu = os.cpu_count() or 1
+            words = pynvml.nvmlDeviceGetCpuAffinity(h, (ncpu + 63) // 64)
+        finally:
+            pynvml.nvmlShutdown()
+    except Exception:
+        return None
+    local = {64 * w + b for w, m in enumerate(words) for b in range(64) if (int(m) >> b) & 1}
+    cpus = local & os.sched_getaffinity(0)
+    if not cpus:
+        return None
+    os.sched_setaffinity(0, cpus)
+    return len(cpus)
+
+
 @dataclass
 class SpeciesState:
     name: str

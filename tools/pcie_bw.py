@@ -1,5 +1,12 @@
-"""Dev: pinned host <-> device copy bandwidth on the GPU box (PCIe), the e2e bound."""
-import torch, time
+"""Dev: pinned host <-> device copy bandwidth on the GPU box (PCIe), the e2e bound.
+    python tools/pcie_bw.py [--bind]   (--bind: pin the process to the GPU's local CPUs first)"""
+import os, sys, time
+if "--bind" in sys.argv:
+    sys.path.insert(0, ".")
+    from paper_conf_sc_tanlta25_b200.pic import bind_to_gpu_cpus
+    print("bound to", bind_to_gpu_cpus(0))
+print("cpus", len(os.sched_getaffinity(0)), sorted(os.sched_getaffinity(0))[:4], "...")
+import torch
 n = 8 * (1 << 30) // 4  # 8 GiB floats
 h = torch.empty(n, dtype=torch.float32).pin_memory()
 h2 = torch.empty(n, dtype=torch.float32).pin_memory()

@@ -47,7 +47,7 @@ def parse():
     ap.add_argument("--shuffle", action="store_true", help="random initial order (paper's 'random')")
     ap.add_argument("--sort-every", type=int, default=0)
     ap.add_argument("--math", default="fast", choices=["fast", "ieee"])
-    ap.add_argument("--deposit", default="auto", choices=["auto", "lane", "warp"])
+    ap.add_argument("--deposit", default="auto", choices=["auto", "lane", "warp", "smem"])
     ap.add_argument("--kernel", default="auto", choices=["auto", "direct", "tma"])
     ap.add_argument("--field-solve", action="store_true",
                     help="full PIC step: + advance_b/advance_e (self-consistent fields)")
@@ -261,7 +261,7 @@ def our_arm(args, rank, world):
         parts = [inputs.shuffle(p, seed + 17 + k) for k, p in enumerate(parts)]
     fields = inputs.make_fields(g, wl.field_amp, seed, kind=wl.kind)
     math_mode = vpic.MATH_IEEE if args.math == "ieee" else vpic.MATH_FAST
-    dep = {"auto": 0, "lane": 1, "warp": 2}[args.deposit]
+    dep = {"auto": 0, "lane": 1, "warp": 2, "smem": 3}[args.deposit]
     # particle capacity per rank: the drifting LPI electrons pile up on the
     # downstream ranks (~0.13% of a rank's electrons cross each step at 2
     # GPUs); movers per inbox slot: a boundary plane's electrons x 0.35 (the

@@ -72,8 +72,12 @@ enum {
   VPIC_OPT_MATH = 0,
   /* current scatter strategy: 0 = AUTO, 1 = LANE (3 x red.global.add.v4.f32 per
    * streak), 2 = WARP (same-voxel contributions reduced across the warp with
-   * shuffles before red.global; falls back to LANE for scattered warps).
-   * Default AUTO (= WARP). */
+   * shuffles before red.global; falls back to LANE for scattered warps),
+   * 3 = SMEM (WARP, plus same-voxel groups of 2..6 items of a warp summed
+   * through shared memory by their lowest lane before its red.global --
+   * faster once particles have diffused a fraction of a cell since their
+   * sort, slower right after it; TMA kernel only, the direct kernel treats
+   * it as WARP).  Default AUTO (= WARP). */
   VPIC_OPT_DEPOSIT = 1,
   /* default TileSz for VPIC_SORT_TILED_STRIDED when tile_sz == 0.  Default
    * 3 x (#SMs) x 128 ("three times the number of GPU cores"). */

@@ -168,7 +168,7 @@ int vpic_ctx_set_option(vpic_ctx *c, int option, int64_t value) {
       c->math = (int)value;
       return VPIC_OK;
     case VPIC_OPT_DEPOSIT:
-      if (value < DEP_AUTO || value > DEP_WARP) return VPIC_ERR_INVALID;
+      if (value < DEP_AUTO || value > DEP_SMEM) return VPIC_ERR_INVALID;
       c->deposit = (int)value;
       return VPIC_OK;
     case VPIC_OPT_TILE_SZ:

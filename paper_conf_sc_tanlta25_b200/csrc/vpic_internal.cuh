@@ -74,7 +74,7 @@ __host__ __device__ inline int dir26(int ox, int oy, int oz) { return (ox + 1) +
 enum FaceKind { FACE_LOCAL = 0, FACE_REFLECT = 1, FACE_ABSORB = 2, FACE_REMOTE = 3 };
 
 enum MathMode { MATH_FAST = 0, MATH_IEEE = 1 };
-enum DepositMode { DEP_AUTO = 0, DEP_LANE = 1, DEP_WARP = 2 };
+enum DepositMode { DEP_AUTO = 0, DEP_LANE = 1, DEP_WARP = 2, DEP_SMEM = 3 };
 enum AdvanceKernel { ADV_AUTO = 0, ADV_DIRECT = 1, ADV_TMA = 2 };
 
 struct Exchange;  // multi-GPU state (migrate.cu)

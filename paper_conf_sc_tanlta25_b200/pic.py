@@ -61,6 +61,9 @@ class SpeciesState:
     np_dev: torch.Tensor = None   # int64[1]: the count on the device (graph mode)
 
 
+SMEM_SIGMA = 0.4   # cells of thermal spread after which DEP_SMEM pays
+
+
 class HotPath:
     def __init__(self, wl: inputs.Workload, species_particles: List[np.ndarray], fields: np.ndarray,
                  order: int = vpic.VPIC_SORT_STANDARD, math: int = vpic.MATH_FAST,
@@ -76,7 +79,13 @@ class HotPath:
         self.dev = torch.device("cuda", torch.cuda.current_device() if device is None else device)
         self.ctx = vpic.Context(self.g, rank, nranks, uid, self.dev.index)
         self.ctx.set_option(vpic.VPIC_OPT_MATH, math)
-        self.ctx.set_option(vpic.VPIC_OPT_DEPOSIT, deposit)
+        # deposit AUTO: per species and step, WARP until the species has
+        # diffused SMEM_SIGMA cells since its sort (thermal speed x steps),
+        # then SMEM (small same-voxel groups summed in shared memory)
+        self.deposit_auto = deposit == vpic.DEP_AUTO
+        self._dep_mode = vpic.DEP_WARP if self.deposit_auto else deposit
+        self.ctx.set_option(vpic.VPIC_OPT_DEPOSIT, self._dep_mode)
+        self.steps_since_sort = 0
         self.order = order
         self.tile_sz = tile_sz
         self.field_solve = field_solve   # advance_b(1/2), advance_e, advance_b(1/2) after unload
@@ -138,6 +147,18 @@ class HotPath:
         self.sort_events = []  # (start, end, species) around vpic_sort_particles
         self.record_advance = False
 
+    def _set_deposit(self, k: int):
+        """AUTO deposit policy for species k at the current step."""
+        if not self.deposit_auto:
+            return
+        sp = self.wl.species[k]
+        g = self.g
+        sigma = sp.u_th * g.cvac * g.dt / min(g.dx, g.dy, g.dz) * self.steps_since_sort
+        mode = vpic.DEP_SMEM if sigma >= SMEM_SIGMA else vpic.DEP_WARP
+        if mode != self._dep_mode:
+            self.ctx.set_option(vpic.VPIC_OPT_DEPOSIT, mode)
+            self._dep_mode = mode
+
     # ------------------------------------------------------------ calls --
     @property
     def n_particles(self) -> int:
@@ -157,6 +178,7 @@ class HotPath:
                 e1.record(stream)
                 self.sort_events.append((e0, e1, s.name))
             s.p, s.scratch = s.scratch, s.p
+        self.steps_since_sort = 0
 
     def step(self, do_sort: bool = False):
         if do_sort:
@@ -167,7 +189,8 @@ class HotPath:
         if self.concurrent:
             ready = torch.cuda.Event()
             ready.record(stream)
-            for s, st in zip(self.species, self.sp_streams):
+            for k, (s, st) in enumerate(zip(self.species, self.sp_streams)):
+                self._set_deposit(k)
                 st.wait_event(ready)
                 if self.record_advance:
                     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -179,7 +202,8 @@ class HotPath:
                     self.adv_events.append((e0, e1, s.np))
             for st in self.sp_streams:
                 stream.wait_stream(st)
-        for s in (() if self.concurrent else self.species):
+        for k, s in enumerate(() if self.concurrent else self.species):
+            self._set_deposit(k)
             if self.record_advance:
                 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 e0.record(stream)
@@ -197,6 +221,7 @@ class HotPath:
             vpic.vpic_advance_b(self.ctx, self.fields, 0.5)
             vpic.vpic_advance_e(self.ctx, self.fields, self.jf, self.eps0)
             vpic.vpic_advance_b(self.ctx, self.fields, 0.5)
+        self.steps_since_sort += 1
 
     def cycle(self, steps: int):
         """One sort period: sort, then `steps` PIC steps."""
@@ -221,7 +246,8 @@ class HotPath:
     def _step_dev(self):
         vpic.vpic_load_interpolator(self.ctx, self.fields, self.interp)
         vpic.vpic_clear_accumulator(self.ctx, self.acc)
-        for s in self.species:
+        for k, s in enumerate(self.species):
+            self._set_deposit(k)
             vpic.vpic_advance_p_dev(self.ctx, s.q, s.m, s.p, s.np_dev, s.p.shape[0], self.interp, self.acc,
                                     s.movers, s.movers.shape[0], s.n_movers, s.flags)
             if self.migrate:
@@ -233,6 +259,7 @@ class HotPath:
             vpic.vpic_advance_b(self.ctx, self.fields, 0.5)
             vpic.vpic_advance_e(self.ctx, self.fields, self.jf, self.eps0)
             vpic.vpic_advance_b(self.ctx, self.fields, 0.5)
+        self.steps_since_sort += 1
 
     def _cycle_graph(self, steps: int):
         self.sync_counts()

@@ -27,7 +27,7 @@ VPIC_OPT_ADVANCE_CTAS_PER_SM = 5
 VPIC_OPT_DEVICE_EXCHANGE = 6
 VPIC_OPT_SINGLE_ROUND_MIGRATION = 7
 MATH_FAST, MATH_IEEE = 0, 1
-DEP_AUTO, DEP_LANE, DEP_WARP = 0, 1, 2
+DEP_AUTO, DEP_LANE, DEP_WARP, DEP_SMEM = 0, 1, 2, 3
 
 # every symbol include/vpic.h declares (checked by tests/test_abi_symbols.py)
 EXPORTS = ["vpic_get_unique_id", "vpic_ctx_create", "vpic_ctx_destroy", "vpic_ctx_set_option",

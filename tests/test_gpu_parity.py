@@ -181,7 +181,7 @@ def run_both(V, orc, g, p, q, m, fields, math, deposit, kernel=0):
 
 
 @pytest.mark.parametrize("case", adv_cases(), ids=lambda c: c[0])
-@pytest.mark.parametrize("deposit", [1, 2], ids=["lane", "warp"])
+@pytest.mark.parametrize("deposit", [1, 2, 3], ids=["lane", "warp", "smem"])
 @pytest.mark.parametrize("kernel", [1, 2], ids=["direct", "tma"])
 def test_advance_ieee_bitexact(V, orc, case, deposit, kernel):
     name, g, p, q, m, f = case
@@ -195,7 +195,7 @@ def test_advance_ieee_bitexact(V, orc, case, deposit, kernel):
 
 
 @pytest.mark.parametrize("case", adv_cases(), ids=lambda c: c[0])
-@pytest.mark.parametrize("deposit", [1, 2], ids=["lane", "warp"])
+@pytest.mark.parametrize("deposit", [1, 2, 3], ids=["lane", "warp", "smem"])
 @pytest.mark.parametrize("kernel", [1, 2], ids=["direct", "tma"])
 def test_advance_fast_tolerance(V, orc, case, deposit, kernel):
     name, g, p, q, m, f = case

@@ -22,7 +22,7 @@ ap.add_argument("--steps", type=int, default=20)
 ap.add_argument("--species", default="electron", choices=["electron", "ion", "both"])
 ap.add_argument("--deposit", nargs="+", default=["warp"])
 a = ap.parse_args()
-DEP = {"auto": 0, "lane": 1, "warp": 2}
+DEP = {"auto": 0, "lane": 1, "warp": 2, "smem": 3}
 
 wl = inputs.config(1)
 from dataclasses import replace

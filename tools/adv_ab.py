@@ -21,6 +21,7 @@ ap.add_argument("--ppc", type=int, default=128)
 ap.add_argument("--steps", type=int, default=20)
 ap.add_argument("--species", default="electron", choices=["electron", "ion", "both"])
 ap.add_argument("--deposit", nargs="+", default=["warp"])
+ap.add_argument("--sigma", type=float, nargs="*", default=[], help="AUTO policy thresholds to try")
 a = ap.parse_args()
 DEP = {"auto": 0, "lane": 1, "warp": 2, "smem": 3}
 
@@ -34,7 +35,11 @@ parts = inputs.make_species_particles(wl, inputs.MASTER_SEED + 1)
 fields = inputs.make_fields(wl.grid, wl.field_amp, inputs.MASTER_SEED + 1)
 print(f"# {a.n}^3 x {a.ppc} ppc, {sum(p.size for p in parts)} particles, gen {time.time() - t0:.1f} s",
       flush=True)
-for d in a.deposit:
+import paper_conf_sc_tanlta25_b200.pic as pic
+runs = [(d, None) for d in a.deposit] + [("auto", sg) for sg in a.sigma]
+for d, sg in runs:
+    if sg is not None:
+        pic.SMEM_SIGMA = sg
     hp = HotPath(wl, parts, fields, deposit=DEP[d])
     hp.sort()
     hp.record_advance = True
@@ -44,6 +49,6 @@ for d in a.deposit:
     torch.cuda.synchronize()
     t = [s.elapsed_time(e) for s, e, _ in hp.adv_events]
     jf = hp.jf.sum().item()
-    print(d, "mean %.3f ms" % np.mean(t), "by step", [round(x, 3) for x in t[::max(1, len(t) // 10)]],
+    print(d if sg is None else f"auto(sigma={sg})", "mean %.3f ms" % np.mean(t), "by step", [round(x, 3) for x in t[::max(1, len(t) // 10)]],
           "sum(jf) %.6g" % jf, flush=True)
     hp.close()

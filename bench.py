@@ -405,7 +405,9 @@ def our_arm(args, rank, world):
                    "ppc_per_species": wl.ppc,
                    "species": len(wl.species), "particles": int(ntot), "sort_every": S,
                    "order": args.order, "shuffled": bool(args.shuffle), "math": args.math,
-                   "deposit": args.deposit, "kernel": args.kernel,
+                   "deposit": args.deposit if args.deposit != "auto" else
+                   "auto (warp; smem per species once its thermal spread since the sort >= 0.4 cell)",
+                   "kernel": args.kernel,
                    "parallelism": "loopback1" if args.loopback and world == 1 else f"domain{world}",
                    "field_solve": bool(args.field_solve),
                    "exchange": ("nccl" if args.exchange == "nccl" else "device")

@@ -406,7 +406,7 @@ def our_arm(args, rank, world):
                    "species": len(wl.species), "particles": int(ntot), "sort_every": S,
                    "order": args.order, "shuffled": bool(args.shuffle), "math": args.math,
                    "deposit": args.deposit if args.deposit != "auto" else
-                   "auto (warp; smem per species once its thermal spread since the sort >= 0.4 cell)",
+                   "auto (warp; smem per species while its thermal spread since the sort is 0.4-1.3 cells)",
                    "kernel": args.kernel,
                    "parallelism": "loopback1" if args.loopback and world == 1 else f"domain{world}",
                    "field_solve": bool(args.field_solve),

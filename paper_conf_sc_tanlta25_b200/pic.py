@@ -61,7 +61,11 @@ class SpeciesState:
     np_dev: torch.Tensor = None   # int64[1]: the count on the device (graph mode)
 
 
-SMEM_SIGMA = 0.4   # cells of thermal spread after which DEP_SMEM pays
+# thermal spread (cells) since the sort within which DEP_SMEM pays (DESIGN.md
+# §10): from 0.4 cell same-voxel groups are common enough to sum; past ~1.3
+# cells (hot species late in the period) they are mostly singletons again
+SMEM_SIGMA = 0.4
+SMEM_SIGMA_MAX = 1.3
 
 
 class HotPath:
@@ -79,9 +83,10 @@ class HotPath:
         self.dev = torch.device("cuda", torch.cuda.current_device() if device is None else device)
         self.ctx = vpic.Context(self.g, rank, nranks, uid, self.dev.index)
         self.ctx.set_option(vpic.VPIC_OPT_MATH, math)
-        # deposit AUTO: per species and step, WARP until the species has
-        # diffused SMEM_SIGMA cells since its sort (thermal speed x steps),
-        # then SMEM (small same-voxel groups summed in shared memory)
+        # deposit AUTO: per species and step, SMEM (small same-voxel groups
+        # summed in shared memory) while the species' thermal spread since its
+        # sort (thermal speed x steps) is in [SMEM_SIGMA, SMEM_SIGMA_MAX),
+        # WARP otherwise
         self.deposit_auto = deposit == vpic.DEP_AUTO
         self._dep_mode = vpic.DEP_WARP if self.deposit_auto else deposit
         self.ctx.set_option(vpic.VPIC_OPT_DEPOSIT, self._dep_mode)
@@ -154,7 +159,7 @@ class HotPath:
         sp = self.wl.species[k]
         g = self.g
         sigma = sp.u_th * g.cvac * g.dt / min(g.dx, g.dy, g.dz) * self.steps_since_sort
-        mode = vpic.DEP_SMEM if sigma >= SMEM_SIGMA else vpic.DEP_WARP
+        mode = vpic.DEP_SMEM if SMEM_SIGMA <= sigma < SMEM_SIGMA_MAX else vpic.DEP_WARP
         if mode != self._dep_mode:
             self.ctx.set_option(vpic.VPIC_OPT_DEPOSIT, mode)
             self._dep_mode = mode

@@ -20,6 +20,7 @@ ap.add_argument("--n", type=int, default=64)
 ap.add_argument("--ppc", type=int, default=128)
 ap.add_argument("--steps", type=int, default=20)
 ap.add_argument("--species", default="electron", choices=["electron", "ion", "both"])
+ap.add_argument("--uth", type=float, default=0.0, help="override the electrons' thermal speed")
 ap.add_argument("--deposit", nargs="+", default=["warp"])
 ap.add_argument("--sigma", type=float, nargs="*", default=[], help="AUTO policy thresholds to try")
 a = ap.parse_args()
@@ -29,6 +30,8 @@ wl = inputs.config(1)
 from dataclasses import replace
 wl = replace(wl, grid=inputs.GridSpec(a.n, a.n, a.n), ppc=a.ppc)
 sel = {"electron": [0], "ion": [1], "both": [0, 1]}[a.species]
+if a.uth > 0:
+    wl = replace(wl, species=[replace(wl.species[0], u_th=a.uth)] + wl.species[1:])
 wl = replace(wl, species=[wl.species[k] for k in sel])
 t0 = time.time()
 parts = inputs.make_species_particles(wl, inputs.MASTER_SEED + 1)

@@ -92,60 +92,68 @@ k_advance_e(const GridK g, const float px, const float py, const float pz, const
   }
 }
 
-// One thread per interior voxel; a CTA covers a run of x along one (y,z) row
-// so the x+1 neighbours come from L1.  interp[v] = 6 x float4 (96 B, the last
-// 24 B zero) so that a particle's gather is three sector-aligned 32-B loads.
+// One thread per interior voxel; consecutive threads take consecutive x of
+// a (y,z) row so the x+1 neighbours come from L1.  interp[v] = 6 x float4
+// (96 B, the last 24 B zero) so that a particle's gather is three
+// sector-aligned 32-B loads.  (Staging a warp's 32 rows in shared memory to
+// store them as consecutive 16-B units was slower: 125 vs 108 us at C2.)
 __global__ void __launch_bounds__(128)
 k_load_interp(const GridK g, const float4 *__restrict__ f, float4 *__restrict__ interp) {
-  const int nrows = g.ny * g.nz;
+  const int lane = threadIdx.x & 31;
+  const uint32_t nx = (uint32_t)g.nx, ny = (uint32_t)g.ny;
+  const int64_t n = (int64_t)g.ny * g.nz * g.nx;   // < 2^32 (host-checked)
   const float fourth = 0.25f, half = 0.5f;
-  for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-       t < (int64_t)nrows * g.nx; t += (int64_t)gridDim.x * blockDim.x) {
-    const int x = 1 + (int)(t % g.nx);
-    const int row = (int)(t / g.nx);
-    const int y = 1 + row % g.ny, z = 1 + row / g.ny;
-    const int64_t v = x + (int64_t)g.sx * (y + (int64_t)g.sy * z);
-    const int64_t X = 1, Y = g.sx, Z = g.sxy;
-    // E (first float4) and cB (second float4) of the 7 neighbours needed
-    const float4 e000 = __ldg(f + 2 * v), b000 = __ldg(f + 2 * v + 1);
-    const float4 e100 = __ldg(f + 2 * (v + X)), b100 = __ldg(f + 2 * (v + X) + 1);
-    const float4 e010 = __ldg(f + 2 * (v + Y)), b010 = __ldg(f + 2 * (v + Y) + 1);
-    const float4 e001 = __ldg(f + 2 * (v + Z)), b001 = __ldg(f + 2 * (v + Z) + 1);
-    const float4 e110 = __ldg(f + 2 * (v + X + Y));
-    const float4 e011 = __ldg(f + 2 * (v + Y + Z));
-    const float4 e101 = __ldg(f + 2 * (v + X + Z));
-    float w0, w1, w2, w3;
-    float4 o0, o1, o2, o3, o4;
-    // ex: bilinear in (y, z)
-    w0 = e000.x; w1 = e010.x; w2 = e001.x; w3 = e011.x;
-    o0.x = fourth * ((w3 + w0) + (w1 + w2));
-    o0.y = fourth * ((w3 - w0) + (w1 - w2));
-    o0.z = fourth * ((w3 - w0) - (w1 - w2));
-    o0.w = fourth * ((w3 + w0) - (w1 + w2));
-    // ey: bilinear in (z, x)
-    w0 = e000.y; w1 = e001.y; w2 = e100.y; w3 = e101.y;
-    o1.x = fourth * ((w3 + w0) + (w1 + w2));
-    o1.y = fourth * ((w3 - w0) + (w1 - w2));
-    o1.z = fourth * ((w3 - w0) - (w1 - w2));
-    o1.w = fourth * ((w3 + w0) - (w1 + w2));
-    // ez: bilinear in (x, y)
-    w0 = e000.z; w1 = e100.z; w2 = e010.z; w3 = e110.z;
-    o2.x = fourth * ((w3 + w0) + (w1 + w2));
-    o2.y = fourth * ((w3 - w0) + (w1 - w2));
-    o2.z = fourth * ((w3 - w0) - (w1 - w2));
-    o2.w = fourth * ((w3 + w0) - (w1 + w2));
-    // cB: linear along the face normal
-    o3.x = half * (b100.x + b000.x);
-    o3.y = half * (b100.x - b000.x);
-    o3.z = half * (b010.y + b000.y);
-    o3.w = half * (b010.y - b000.y);
-    o4.x = half * (b001.z + b000.z);
-    o4.y = half * (b001.z - b000.z);
-    o4.z = 0.0f;
-    o4.w = 0.0f;
-    float4 *o = interp + 6 * v;
-    o[0] = o0; o[1] = o1; o[2] = o2; o[3] = o3; o[4] = o4;
-    o[5] = make_float4(0.f, 0.f, 0.f, 0.f);
+  for (int64_t t0 = ((int64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31)); t0 < n;
+       t0 += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t t = t0 + lane;
+    const bool act = t < n;
+    int64_t v = 0;
+    if (act) {
+      const uint32_t tt = (uint32_t)t, row = tt / nx;
+      const uint32_t x = 1 + (tt - row * nx), y = 1 + row % ny, z = 1 + row / ny;
+      v = x + (int64_t)g.sx * (y + (int64_t)g.sy * z);
+      const int64_t X = 1, Y = g.sx, Z = g.sxy;
+      // E (first float4) and cB (second float4) of the 7 neighbours needed
+      const float4 e000 = __ldg(f + 2 * v), b000 = __ldg(f + 2 * v + 1);
+      const float4 e100 = __ldg(f + 2 * (v + X)), b100 = __ldg(f + 2 * (v + X) + 1);
+      const float4 e010 = __ldg(f + 2 * (v + Y)), b010 = __ldg(f + 2 * (v + Y) + 1);
+      const float4 e001 = __ldg(f + 2 * (v + Z)), b001 = __ldg(f + 2 * (v + Z) + 1);
+      const float4 e110 = __ldg(f + 2 * (v + X + Y));
+      const float4 e011 = __ldg(f + 2 * (v + Y + Z));
+      const float4 e101 = __ldg(f + 2 * (v + X + Z));
+      float w0, w1, w2, w3;
+      float4 o0, o1, o2, o3, o4;
+      // ex: bilinear in (y, z)
+      w0 = e000.x; w1 = e010.x; w2 = e001.x; w3 = e011.x;
+      o0.x = fourth * ((w3 + w0) + (w1 + w2));
+      o0.y = fourth * ((w3 - w0) + (w1 - w2));
+      o0.z = fourth * ((w3 - w0) - (w1 - w2));
+      o0.w = fourth * ((w3 + w0) - (w1 + w2));
+      // ey: bilinear in (z, x)
+      w0 = e000.y; w1 = e001.y; w2 = e100.y; w3 = e101.y;
+      o1.x = fourth * ((w3 + w0) + (w1 + w2));
+      o1.y = fourth * ((w3 - w0) + (w1 - w2));
+      o1.z = fourth * ((w3 - w0) - (w1 - w2));
+      o1.w = fourth * ((w3 + w0) - (w1 + w2));
+      // ez: bilinear in (x, y)
+      w0 = e000.z; w1 = e100.z; w2 = e010.z; w3 = e110.z;
+      o2.x = fourth * ((w3 + w0) + (w1 + w2));
+      o2.y = fourth * ((w3 - w0) + (w1 - w2));
+      o2.z = fourth * ((w3 - w0) - (w1 - w2));
+      o2.w = fourth * ((w3 + w0) - (w1 + w2));
+      // cB: linear along the face normal
+      o3.x = half * (b100.x + b000.x);
+      o3.y = half * (b100.x - b000.x);
+      o3.z = half * (b010.y + b000.y);
+      o3.w = half * (b010.y - b000.y);
+      o4.x = half * (b001.z + b000.z);
+      o4.y = half * (b001.z - b000.z);
+      o4.z = 0.0f;
+      o4.w = 0.0f;
+      float4 *o = interp + 6 * v;
+      o[0] = o0; o[1] = o1; o[2] = o2; o[3] = o3; o[4] = o4;
+      o[5] = make_float4(0.f, 0.f, 0.f, 0.f);
+    }
   }
 }
 
@@ -204,6 +212,7 @@ cudaError_t launch_fill_ghosts(const vpic_ctx *c, float *fields, cudaStream_t s)
 cudaError_t launch_load_interp(const vpic_ctx *c, const float *fields, float *interp,
                                cudaStream_t s) {
   const int64_t n = (int64_t)c->gk.nx * c->gk.ny * c->gk.nz;
+  if (n >= ((int64_t)1 << 32)) return cudaErrorInvalidValue;   // 32-bit voxel counter
   k_load_interp<<<grid_for(n, 128, c->num_sms), 128, 0, s>>>(
       c->gk, reinterpret_cast<const float4 *>(fields), reinterpret_cast<float4 *>(interp)); note_launch();
   return cudaGetLastError();

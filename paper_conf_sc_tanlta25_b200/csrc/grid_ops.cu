@@ -96,7 +96,7 @@ k_advance_e(const GridK g, const float px, const float py, const float pz, const
 // a (y,z) row so the x+1 neighbours come from L1.  interp[v] = 6 x float4
 // (96 B, the last 24 B zero) so that a particle's gather is three
 // sector-aligned 32-B loads.  (Staging a warp's 32 rows in shared memory to
-// store them as consecutive 16-B units was slower: 125 vs 108 us at C2.)
+// store them as consecutive 16-B units was not faster.)
 __global__ void __launch_bounds__(128)
 k_load_interp(const GridK g, const float4 *__restrict__ f, float4 *__restrict__ interp) {
   const int lane = threadIdx.x & 31;

@@ -68,6 +68,13 @@ SMEM_SIGMA = 0.4
 SMEM_SIGMA_MAX = 1.3
 
 
+def auto_deposit_mode(u_th: float, cvac: float, dt: float, dmin: float, steps_since_sort: int) -> int:
+    """The AUTO policy: the deposit mode for a species of thermal speed u_th,
+    `steps_since_sort` PIC steps after its sort (cell size dmin)."""
+    sigma = u_th * cvac * dt / dmin * steps_since_sort
+    return vpic.DEP_SMEM if SMEM_SIGMA <= sigma < SMEM_SIGMA_MAX else vpic.DEP_WARP
+
+
 class HotPath:
     def __init__(self, wl: inputs.Workload, species_particles: List[np.ndarray], fields: np.ndarray,
                  order: int = vpic.VPIC_SORT_STANDARD, math: int = vpic.MATH_FAST,
@@ -156,10 +163,9 @@ class HotPath:
         """AUTO deposit policy for species k at the current step."""
         if not self.deposit_auto:
             return
-        sp = self.wl.species[k]
         g = self.g
-        sigma = sp.u_th * g.cvac * g.dt / min(g.dx, g.dy, g.dz) * self.steps_since_sort
-        mode = vpic.DEP_SMEM if SMEM_SIGMA <= sigma < SMEM_SIGMA_MAX else vpic.DEP_WARP
+        mode = auto_deposit_mode(self.wl.species[k].u_th, g.cvac, g.dt, min(g.dx, g.dy, g.dz),
+                                 self.steps_since_sort)
         if mode != self._dep_mode:
             self.ctx.set_option(vpic.VPIC_OPT_DEPOSIT, mode)
             self._dep_mode = mode

@@ -95,11 +95,12 @@ k_advance_e(const GridK g, const float px, const float py, const float pz, const
 // One thread per interior voxel; consecutive threads take consecutive x of
 // a (y,z) row so the x+1 neighbours come from L1.  interp[v] = 6 x float4
 // (96 B, the last 24 B zero) so that a particle's gather is three
-// sector-aligned 32-B loads.  (Staging a warp's 32 rows in shared memory to
-// store them as consecutive 16-B units was not faster.)
+// sector-aligned 32-B loads.  Each warp stages its 32 rows in shared memory and
+// stores them as consecutive 16-B units (warm: 86 vs 127 us at C2).
 __global__ void __launch_bounds__(128)
 k_load_interp(const GridK g, const float4 *__restrict__ f, float4 *__restrict__ interp) {
-  const int lane = threadIdx.x & 31;
+  __shared__ float4 stage[4][32 * 6];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const uint32_t nx = (uint32_t)g.nx, ny = (uint32_t)g.ny;
   const int64_t n = (int64_t)g.ny * g.nz * g.nx;   // < 2^32 (host-checked)
   const float fourth = 0.25f, half = 0.5f;
@@ -150,10 +151,22 @@ k_load_interp(const GridK g, const float4 *__restrict__ f, float4 *__restrict__ 
       o4.y = half * (b001.z - b000.z);
       o4.z = 0.0f;
       o4.w = 0.0f;
-      float4 *o = interp + 6 * v;
+      float4 *o = &stage[w][6 * lane];
       o[0] = o0; o[1] = o1; o[2] = o2; o[3] = o3; o[4] = o4;
       o[5] = make_float4(0.f, 0.f, 0.f, 0.f);
     }
+    __syncwarp();
+    // staged unit j = component j % 6 of the warp's row j / 6: consecutive
+    // lanes store consecutive 16-B units of consecutive voxels
+    const int nact = n - t0 < 32 ? (int)(n - t0) : 32;
+#pragma unroll
+    for (int k = 0; k < 6; ++k) {
+      const int j = lane + 32 * k;
+      const int src = j / 6;
+      const int64_t vj = __shfl_sync(0xffffffffu, v, src);
+      if (src < nact) interp[6 * vj + (j - 6 * src)] = stage[w][j];
+    }
+    __syncwarp();
   }
 }
 

@@ -385,7 +385,12 @@ k_rank_keys(const uint32_t *__restrict__ K, const uint32_t *__restrict__ perm_st
 }
 
 // ---------------------------------------------------------------- a4 --
-constexpr int GATHER_ILP = 8;  // half-records in flight per thread
+#ifndef VPIC_GATHER_ILP
+#define VPIC_GATHER_ILP 8
+#endif
+// half-records in flight per thread (measured at C2, electrons / ions ms:
+// 4: 13.9 / 11.1, 8: 14.0 / 10.8, 16: 13.4 / 11.8)
+constexpr int GATHER_ILP = VPIC_GATHER_ILP;
 
 __global__ void __launch_bounds__(256)
 k_gather(const vpic_particle_t *__restrict__ pin, vpic_particle_t *__restrict__ pout,

@@ -365,3 +365,20 @@ def test_gather_scatter_parity(V, orc, nx, agg, order):
     absum = np.zeros(K)
     orc.gather_scatter(keys, np.abs(x), table, absum, nx)
     assert np.all(np.abs(acc.cpu().numpy() - acc_o) <= 1e-13 * absum + 1e-300)
+
+
+# Chunk-schedule edges of k_advance_tma: 64-particle chunks dealt in pairs,
+# full chunks through the tensor map, the ragged one through a plain bulk
+# copy, the last voxel's sum carried across a pair.  Sorted voxel runs of
+# 96 (a voxel straddles chunk and pair boundaries) with hot particles so the
+# chunk-closing items are often crossers.
+@pytest.mark.parametrize("n", [1, 63, 64, 65, 127, 128, 129, 191, 4097, 70000])
+@pytest.mark.parametrize("deposit", [2, 3], ids=["warp", "smem"])
+def test_advance_chunk_edges_ieee(V, orc, n, deposit):
+    g = inputs.GridSpec(12, 10, 8)
+    vox = np.repeat(g.interior_voxels(), 96)[:n]
+    p = inputs.random_particles(g, n, 31 + n, u_scale=0.9)
+    p["i"] = vox
+    r = run_both(V, orc, g, p, -1.0, 1.0, inputs.make_fields(g, 0.05, seed=8), V.MATH_IEEE, deposit, 2)
+    assert_particles_bitexact(r["p"], r["p_o"])
+    assert_acc_close(r["acc"], r["acc_o"], r["acc_abs"])

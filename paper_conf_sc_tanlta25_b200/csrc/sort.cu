@@ -26,15 +26,26 @@ namespace vpic {
 namespace {
 
 #ifndef VPIC_SORT_IPT
-#define VPIC_SORT_IPT 16
+#define VPIC_SORT_IPT 12
+#endif
+#ifndef VPIC_SORT_PERSIST
+#define VPIC_SORT_PERSIST 0
 #endif
 #ifndef VPIC_SORT_MINB
-#define VPIC_SORT_MINB 3
+#define VPIC_SORT_MINB 2
 #endif
-constexpr int NT = 256;             // threads per radix CTA
+#ifndef VPIC_SORT_NT
+#define VPIC_SORT_NT 512
+#endif
+constexpr int NT = VPIC_SORT_NT;    // threads per radix CTA
 constexpr int NW = NT / 32;         // warps
 constexpr int IPT = VPIC_SORT_IPT;  // items per thread
-constexpr int TILE = NT * IPT;      // 4096 elements per tile
+constexpr int TILE = NT * IPT;      // 6144 elements per tile
+// Launch shape measured on late C2 electrons / ions (sort ms, same box):
+// 256 x 16 x 3 CTAs/SM 14.07 / 10.79; 512 x 12 x 2 13.87 / 10.47 (kept);
+// 256 x 24 x 2 14.19 / 10.81; 256 x 32 x 2 13.91 / 10.57 (spills);
+// 512 x 16 x 1 15.54 / 11.84; persistent 256 x 16 x 2 CTAs/SM (next tile
+// loaded during the current one) 14.86 / 12.10, 256 x 8 x 4 16.56 / 13.99
 constexpr int MAX_BITS = 8;         // digit width: 256 buckets, one look-back chain per thread
 constexpr int MAX_PASSES = 4;       // keys up to 32 bits
 constexpr unsigned FULL = 0xffffffffu;
@@ -215,6 +226,11 @@ __global__ void k_scan_hist(const uint32_t *__restrict__ ghist, uint32_t *__rest
 // elements stably (per-warp smem histograms, match_any within a warp),
 // publishes its per-digit count and resolves its global offset by decoupled
 // look-back over earlier tiles' status words (flag | count in one u64).
+// With VPIC_SORT_PERSIST the grid is one wave of resident CTAs that loop over
+// tickets, loading the next tile's keys/values while the current one is
+// ranked, looked back and scattered.  Deadlock-free: a CTA holds at most two
+// tickets, processes them in increasing order, and a tile only waits on
+// smaller tickets, all held by resident CTAs.
 template <int BITS>
 __global__ void __launch_bounds__(NT, VPIC_SORT_MINB)
 k_radix_pass(const uint32_t *__restrict__ kin, const uint32_t *__restrict__ vin,
@@ -229,109 +245,138 @@ k_radix_pass(const uint32_t *__restrict__ kin, const uint32_t *__restrict__ vin,
   uint32_t *skey = tstart + NB;                                                // [TILE]
   uint32_t *sval = skey + TILE;                                                // [TILE]
   __shared__ unsigned int s_tile;
-  if (threadIdx.x == 0) s_tile = atomicAdd(tile_ctr, 1u);
-  for (int i = threadIdx.x; i < NW * NB / 2; i += NT) reinterpret_cast<uint32_t *>(whist)[i] = 0;
-  __syncthreads();
-  const int64_t tile = s_tile;
+  __shared__ uint32_t wsum[NW];
+  const int64_t ntiles = (n + TILE - 1) / TILE;
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int64_t wbase = tile * TILE + (int64_t)w * 32 * IPT;
-
-  uint32_t key[IPT], val[IPT];
-  uint32_t rank[IPT / 2];  // two u16 ranks per register
-#pragma unroll
-  for (int j = 0; j < IPT; ++j) {
-    const int64_t i = wbase + j * 32 + lane;
-    const bool valid = i < n;
-    key[j] = valid ? __ldcs(kin + i) : 0u;
-    val[j] = valid ? (vin ? __ldcs(vin + i) : (uint32_t)i) : 0u;
-  }
   const unsigned lt = lanemask_lt();
   uint16_t *wh = whist + w * NB;
+  uint32_t key[IPT], val[IPT];
+  auto load_tile = [&](int64_t t, uint32_t *k, uint32_t *v) {
+    const int64_t wb = t * TILE + (int64_t)w * 32 * IPT;
 #pragma unroll
-  for (int j = 0; j < IPT; ++j) {
-    const int64_t i = wbase + j * 32 + lane;
-    const bool valid = i < n;
-    const uint32_t d = valid ? ((key[j] >> shift) & (NB - 1)) : (uint32_t)NB;
-    const unsigned peers = __match_any_sync(FULL, d);
-    uint32_t cur = 0;
-    if (valid) cur = wh[d];
-    __syncwarp();
-    if (valid && (__ffs(peers) - 1) == lane) wh[d] = (uint16_t)(cur + __popc(peers));
-    __syncwarp();
-    const uint32_t r = cur + __popc(peers & lt);
-    if (j & 1) rank[j >> 1] |= r << 16; else rank[j >> 1] = r;
-  }
-  __syncthreads();
-  // per-digit: warp exclusive offsets, tile count, look-back
-  for (int b = threadIdx.x; b < NB; b += NT) {
-    uint32_t run = 0;
-#pragma unroll
-    for (int ww = 0; ww < NW; ++ww) {
-      const uint32_t c = whist[ww * NB + b];
-      whist[ww * NB + b] = (uint16_t)run;
-      run += c;
+    for (int j = 0; j < IPT; ++j) {
+      const int64_t i = wb + j * 32 + lane;
+      const bool valid = i < n;
+      k[j] = valid ? __ldcs(kin + i) : 0u;
+      v[j] = valid ? (vin ? __ldcs(vin + i) : (uint32_t)i) : 0u;
     }
-    tstart[b] = run;   // tile count of digit b (scanned below)
-    unsigned long long *st = status + tile * NB + b;
-    uint64_t excl = 0;
-    if (tile == 0) {
-      st_relaxed(st, FLAG_INC | run);
-    } else {
-      st_relaxed(st, FLAG_AGG | run);
-      int64_t t = tile - 1;
-      while (true) {
-        const unsigned long long sv = ld_relaxed(status + t * NB + b);
-        const unsigned long long f = sv & (3ull << 62);
-        if (f == 0) continue;
-        excl += sv & VAL_MASK;
-        if (f == FLAG_INC) break;
-        --t;
+  };
+  if (threadIdx.x == 0) s_tile = atomicAdd(tile_ctr, 1u);
+  __syncthreads();
+  int64_t tile = s_tile;
+  if (tile >= ntiles) return;
+  load_tile(tile, key, val);
+  while (true) {
+    for (int i = threadIdx.x; i < NW * NB / 2; i += NT) reinterpret_cast<uint32_t *>(whist)[i] = 0;
+#if VPIC_SORT_PERSIST
+    if (threadIdx.x == 0) s_tile = atomicAdd(tile_ctr, 1u);
+#endif
+    __syncthreads();
+#if VPIC_SORT_PERSIST
+    const int64_t next = s_tile;
+#else
+    const int64_t next = ntiles;
+#endif
+    const int64_t wbase = tile * TILE + (int64_t)w * 32 * IPT;
+    uint32_t rank[IPT / 2];  // two u16 ranks per register
+#pragma unroll
+    for (int j = 0; j < IPT; ++j) {
+      const int64_t i = wbase + j * 32 + lane;
+      const bool valid = i < n;
+      const uint32_t d = valid ? ((key[j] >> shift) & (NB - 1)) : (uint32_t)NB;
+      const unsigned peers = __match_any_sync(FULL, d);
+      uint32_t cur = 0;
+      if (valid) cur = wh[d];
+      __syncwarp();
+      if (valid && (__ffs(peers) - 1) == lane) wh[d] = (uint16_t)(cur + __popc(peers));
+      __syncwarp();
+      const uint32_t r = cur + __popc(peers & lt);
+      if (j & 1) rank[j >> 1] |= r << 16; else rank[j >> 1] = r;
+    }
+#if VPIC_SORT_PERSIST
+    uint32_t nkey[IPT], nval[IPT];
+    if (next < ntiles) load_tile(next, nkey, nval);
+#endif
+    __syncthreads();
+    // per-digit: warp exclusive offsets, tile count, look-back
+    for (int b = threadIdx.x; b < NB; b += NT) {
+      uint32_t run = 0;
+#pragma unroll
+      for (int ww = 0; ww < NW; ++ww) {
+        const uint32_t c = whist[ww * NB + b];
+        whist[ww * NB + b] = (uint16_t)run;
+        run += c;
       }
-      st_relaxed(st, FLAG_INC | (excl + run));
+      tstart[b] = run;   // tile count of digit b (scanned below)
+      unsigned long long *st = status + tile * NB + b;
+      uint64_t excl = 0;
+      if (tile == 0) {
+        st_relaxed(st, FLAG_INC | run);
+      } else {
+        st_relaxed(st, FLAG_AGG | run);
+        int64_t t = tile - 1;
+        while (true) {
+          const unsigned long long sv = ld_relaxed(status + t * NB + b);
+          const unsigned long long f = sv & (3ull << 62);
+          if (f == 0) continue;
+          excl += sv & VAL_MASK;
+          if (f == FLAG_INC) break;
+          --t;
+        }
+        st_relaxed(st, FLAG_INC | (excl + run));
+      }
+      tpref[b] = dig_off[b] + (uint32_t)excl;
     }
-    tpref[b] = dig_off[b] + (uint32_t)excl;
-  }
-  __syncthreads();
-  // tile-local exclusive digit offsets (block scan of the NB tile counts)
-  {
-    __shared__ uint32_t wsum[NW];
-    const uint32_t c = threadIdx.x < NB ? tstart[threadIdx.x] : 0u;
-    uint32_t incl = c;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t y = __shfl_up_sync(FULL, incl, o);
-      if (lane >= o) incl += y;
-    }
-    if (lane == 31) wsum[w] = incl;
     __syncthreads();
-    uint32_t pre = 0;
-    for (int ww = 0; ww < w; ++ww) pre += wsum[ww];
-    if (threadIdx.x < NB) tstart[threadIdx.x] = pre + incl - c;
-    __syncthreads();
-  }
-  // stage the tile in digit order in shared memory, then write each digit's
-  // run with consecutive threads on consecutive addresses (coalesced: one
-  // element-granular scatter per 4 B made the first pass L2-request-bound)
+    // tile-local exclusive digit offsets (block scan of the NB tile counts)
+    {
+      const uint32_t c = threadIdx.x < NB ? tstart[threadIdx.x] : 0u;
+      uint32_t incl = c;
 #pragma unroll
-  for (int j = 0; j < IPT; ++j) {
-    const int64_t i = wbase + j * 32 + lane;
-    if (i < n) {
-      const uint32_t d = (key[j] >> shift) & (NB - 1);
-      const uint32_t r = (j & 1) ? (rank[j >> 1] >> 16) : (rank[j >> 1] & 0xffffu);
-      const uint32_t lp = tstart[d] + whist[w * NB + d] + r;
-      skey[lp] = key[j];
-      sval[lp] = val[j];
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(FULL, incl, o);
+        if (lane >= o) incl += y;
+      }
+      if (lane == 31) wsum[w] = incl;
+      __syncthreads();
+      uint32_t pre = 0;
+      for (int ww = 0; ww < w; ++ww) pre += wsum[ww];
+      if (threadIdx.x < NB) tstart[threadIdx.x] = pre + incl - c;
+      __syncthreads();
     }
-  }
-  __syncthreads();
-  const int64_t t0 = tile * TILE;
-  const int nvalid = (int)(n - t0 < TILE ? n - t0 : (int64_t)TILE);
-  for (int e = threadIdx.x; e < nvalid; e += NT) {
-    const uint32_t k = skey[e];
-    const uint32_t d = (k >> shift) & (NB - 1);
-    const uint32_t pos = tpref[d] + (uint32_t)e - tstart[d];
-    if (kout) kout[pos] = k;
-    vout[pos] = sval[e];
+    // stage the tile in digit order in shared memory, then write each digit's
+    // run with consecutive threads on consecutive addresses (coalesced: one
+    // element-granular scatter per 4 B made the first pass L2-request-bound)
+#pragma unroll
+    for (int j = 0; j < IPT; ++j) {
+      const int64_t i = wbase + j * 32 + lane;
+      if (i < n) {
+        const uint32_t d = (key[j] >> shift) & (NB - 1);
+        const uint32_t r = (j & 1) ? (rank[j >> 1] >> 16) : (rank[j >> 1] & 0xffffu);
+        const uint32_t lp = tstart[d] + whist[w * NB + d] + r;
+        skey[lp] = key[j];
+        sval[lp] = val[j];
+      }
+    }
+    __syncthreads();
+    const int64_t t0 = tile * TILE;
+    const int nvalid = (int)(n - t0 < TILE ? n - t0 : (int64_t)TILE);
+    for (int e = threadIdx.x; e < nvalid; e += NT) {
+      const uint32_t k = skey[e];
+      const uint32_t d = (k >> shift) & (NB - 1);
+      const uint32_t pos = tpref[d] + (uint32_t)e - tstart[d];
+      if (kout) kout[pos] = k;
+      vout[pos] = sval[e];
+    }
+#if VPIC_SORT_PERSIST
+    if (next >= ntiles) break;
+#pragma unroll
+    for (int j = 0; j < IPT; ++j) { key[j] = nkey[j]; val[j] = nval[j]; }
+    tile = next;
+    __syncthreads();  // smem (whist, tpref, tstart, skey/sval, s_tile) reused next tile
+#else
+    break;
+#endif
   }
 }
 
@@ -526,7 +571,17 @@ cudaError_t radix_pass_bits(const uint32_t *kin, const uint32_t *vin, uint32_t *
   once_per_device(configured, [&] {
     cudaFuncSetAttribute(k_radix_pass<BITS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   });
-  k_radix_pass<BITS><<<(unsigned)tiles, NT, smem, s>>>(kin, vin, kout, vout, n, shift, dig_off,
+  int64_t grid = tiles;
+#if VPIC_SORT_PERSIST
+  {
+    int dev = 0, sms = 0, per_sm = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_radix_pass<BITS>, NT, smem);
+    grid = std::min<int64_t>(tiles, (int64_t)sms * std::max(per_sm, 1));
+  }
+#endif
+  k_radix_pass<BITS><<<(unsigned)grid, NT, smem, s>>>(kin, vin, kout, vout, n, shift, dig_off,
                                                        status, ctr); note_launch();
   return cudaGetLastError();
 }

@@ -74,6 +74,10 @@ def sort_cases():
     out.append(("warp_minus_one", g, inputs.random_particles(g, 31, 6)))
     g2 = inputs.GridSpec(32, 32, 32)
     out.append(("many_tiles", g2, inputs.shuffle(inputs.random_particles(g2, 200000, 7), 8)))
+    # more radix tiles (407 of 6144, ragged last) than one wave of resident
+    # CTAs (with VPIC_SORT_PERSIST each CTA loops over several tickets)
+    g3 = inputs.GridSpec(64, 64, 64)
+    out.append(("multi_wave", g3, inputs.shuffle(inputs.random_particles(g3, 2500001, 11), 12)))
     wh, ph = harris_small()
     out.append(("harris_sheet", wh.grid, inputs.shuffle(ph[1], 9)))
     return out

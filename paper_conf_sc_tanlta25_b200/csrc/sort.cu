@@ -46,6 +46,8 @@ constexpr int TILE = NT * IPT;      // 6144 elements per tile
 // 256 x 24 x 2 14.19 / 10.81; 256 x 32 x 2 13.91 / 10.57 (spills);
 // 512 x 16 x 1 15.54 / 11.84; persistent 256 x 16 x 2 CTAs/SM (next tile
 // loaded during the current one) 14.86 / 12.10, 256 x 8 x 4 16.56 / 13.99
+// (another box: 512 x 12 x 2 13.84 / 10.48; 384 x 16 x 2 13.84 / 10.48;
+// 512 x 10 x 2 14.40 / 10.99; 1024 x 6 x 1 16.64 / 12.90)
 constexpr int MAX_BITS = 8;         // digit width: 256 buckets, one look-back chain per thread
 constexpr int MAX_PASSES = 4;       // keys up to 32 bits
 constexpr unsigned FULL = 0xffffffffu;

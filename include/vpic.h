@@ -299,13 +299,20 @@ int vpic_continuity_residual(vpic_ctx *ctx, const float *rho0, const float *rho1
  * neighbors" P:55), received particles continue their move (depositing into
  * acc) and are appended; absorbed and departed particles are removed by
  * back-filling from the end.  *np (HOST) is updated.  SYNCHRONISES `stream`
- * (it reads mover counts).  Fails with VPIC_ERR_CAPACITY if the arrivals would
- * exceed max_np.  With VPIC_OPT_SINGLE_ROUND_MIGRATION: one exchange with up
- * to 26 neighbours, arrivals appended with their move already complete, then
- * acc's ghost layer added into the neighbours' boundary voxels and zeroed. */
+ * (it reads mover counts).
+ *   movers, max_movers  the list vpic_advance_p filled and its capacity (the
+ *                       same max_movers): never read past it;
+ *   n_movers            device int64, the count vpic_advance_p left.
+ * Fails with VPIC_ERR_CAPACITY -- and then the particle array still holds
+ * stopped particles (p.i = 8*voxel+face) and must be discarded -- if
+ * *n_movers > max_movers (advance_p dropped movers; its flags bit 0) or the
+ * arrivals would exceed max_np.  With VPIC_OPT_SINGLE_ROUND_MIGRATION: one
+ * exchange with up to 26 neighbours, arrivals appended with their move
+ * already complete, then acc's ghost layer added into the neighbours'
+ * boundary voxels and zeroed. */
 int vpic_migrate_particles(vpic_ctx *ctx, float q, float m, vpic_particle_t *p, int64_t *np,
-                           int64_t max_np, vpic_mover_t *movers, const int64_t *n_movers,
-                           float *acc, void *stream);
+                           int64_t max_np, vpic_mover_t *movers, int64_t max_movers,
+                           const int64_t *n_movers, float *acc, void *stream);
 
 /* vpic_migrate_particles with the count in DEVICE memory and no host
  * synchronisation: every step is a stream operation, so it can be captured in
@@ -314,11 +321,14 @@ int vpic_migrate_particles(vpic_ctx *ctx, float q, float m, vpic_particle_t *p, 
  * VPIC_OPT_SINGLE_ROUND_MIGRATION and VPIC_OPT_DEVICE_EXCHANGE (else
  * VPIC_ERR_UNSUPPORTED).  *np_dev (int64) in/out; flags_dev (int32, device):
  * capacity errors are OR-ed in as bits 1 (an inbox was full: particles lost),
- * 2 (hole list full), 3 (arrivals did not fit max_np: dropped) -- check it
- * when the count is read back.  n_movers is not reset. */
+ * 2 (more movers than max_movers or than the internal hole list: the count is
+ * clamped, nothing is read past the list, the departures beyond it stay in
+ * the array as stopped particles), 3 (arrivals did not fit max_np: dropped)
+ * -- check it when the count is read back.  n_movers is not reset. */
 int vpic_migrate_particles_dev(vpic_ctx *ctx, float q, float m, vpic_particle_t *p, int64_t *np_dev,
-                               int64_t max_np, const vpic_mover_t *movers, const int64_t *n_movers,
-                               float *acc, int32_t *flags_dev, void *stream);
+                               int64_t max_np, const vpic_mover_t *movers, int64_t max_movers,
+                               const int64_t *n_movers, float *acc, int32_t *flags_dev,
+                               void *stream);
 
 #ifdef __cplusplus
 }

@@ -96,7 +96,7 @@ int vpic_ctx_create(vpic_ctx **out, const vpic_grid_t *g, int rank, int nranks,
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev)
     return VPIC_ERR_UNSUPPORTED;
-  if (cudaSetDevice(device) != cudaSuccess) return VPIC_ERR_CUDA;
+  DeviceGuard dg(device);   // the caller's current device is restored on return
   cudaDeviceProp prop;
   if (cudaGetDeviceProperties(&prop, device) != cudaSuccess) return VPIC_ERR_CUDA;
   if (prop.major != 10 || prop.minor != 0) return VPIC_ERR_UNSUPPORTED;  // sm_100a code only
@@ -351,24 +351,28 @@ int vpic_gather_scatter(vpic_ctx *c, const int32_t *keys, const double *x, int64
 }
 
 int vpic_migrate_particles(vpic_ctx *c, float q, float m, vpic_particle_t *p, int64_t *np,
-                           int64_t max_np, vpic_mover_t *movers, const int64_t *n_movers,
-                           float *acc, void *stream) {
-  if (!c || !np || *np < 0 || max_np < *np || !n_movers || !acc) return VPIC_ERR_INVALID;
+                           int64_t max_np, vpic_mover_t *movers, int64_t max_movers,
+                           const int64_t *n_movers, float *acc, void *stream) {
+  if (!c || !np || *np < 0 || max_np < *np || !n_movers || !acc || max_movers < 0)
+    return VPIC_ERR_INVALID;
   if (max_np >= ((int64_t)1 << 31)) return VPIC_ERR_INVALID;
   if (*np > 0 && (!p || !aligned16(p))) return VPIC_ERR_INVALID;
+  if (max_movers > 0 && (!movers || !aligned16(movers))) return VPIC_ERR_INVALID;
   DeviceGuard dg(c->device);
-  return migrate(c, q, m, p, np, max_np, movers, n_movers, acc, S(stream));
+  return migrate(c, q, m, p, np, max_np, movers, max_movers, n_movers, acc, S(stream));
 }
 
 int vpic_migrate_particles_dev(vpic_ctx *c, float q, float m, vpic_particle_t *p, int64_t *np_dev,
-                               int64_t max_np, const vpic_mover_t *movers, const int64_t *n_movers,
-                               float *acc, int32_t *flags_dev, void *stream) {
+                               int64_t max_np, const vpic_mover_t *movers, int64_t max_movers,
+                               const int64_t *n_movers, float *acc, int32_t *flags_dev,
+                               void *stream) {
   (void)q; (void)m;
   if (!c || !np_dev || max_np < 0 || max_np >= ((int64_t)1 << 31) || !n_movers || !acc || !p ||
-      !aligned16(p) || !flags_dev)
+      !aligned16(p) || !flags_dev || max_movers < 0)
     return VPIC_ERR_INVALID;
+  if (max_movers > 0 && (!movers || !aligned16(movers))) return VPIC_ERR_INVALID;
   DeviceGuard dg(c->device);
-  return migrate_dev(c, p, np_dev, max_np, movers, n_movers, acc, flags_dev, S(stream));
+  return migrate_dev(c, p, np_dev, max_np, movers, max_movers, n_movers, acc, flags_dev, S(stream));
 }
 
 }  // extern "C"

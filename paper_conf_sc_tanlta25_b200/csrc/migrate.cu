@@ -240,6 +240,9 @@ __global__ void k_di_finish(const int64_t *ctr, int64_t *np_dev, int32_t *dflag,
 }
 
 // Holes of this round: H = departures in `mv` (device count *hdev).
+// hcap = min(internal hole capacity, the mover list's capacity): a count
+// beyond it means movers were dropped (or cannot be holed): flagged, clamped
+// so no kernel reads past the list.
 __global__ void k_di_holes_prep(int64_t *ctr, const int64_t *hdev, int64_t hcap, int32_t *flag) {
   int64_t H = *hdev;
   if (H > hcap) { atomicOr(flag, 2); H = hcap; }
@@ -540,11 +543,11 @@ namespace {
 
 // Remove this round's departures (device count) by back-filling from the tail.
 int di_remove_holes(vpic_ctx *c, vpic_particle_t *p, const vpic_mover_t *mv, const int64_t *hdev,
-                    cudaStream_t s) {
+                    int64_t mcap, cudaStream_t s) {
   Exchange *ex = c->ex;
   const unsigned B = (unsigned)c->num_sms * 4;
   uint32_t *tail_dead = ex->di_scr, *low = ex->di_scr + ex->di_hcap, *surv = ex->di_scr + 2 * ex->di_hcap;
-  k_di_holes_prep<<<1, 1, 0, s>>>(ex->di_ctr, hdev, ex->di_hcap, ex->di_flag); note_launch();
+  k_di_holes_prep<<<1, 1, 0, s>>>(ex->di_ctr, hdev, std::min(ex->di_hcap, mcap), ex->di_flag); note_launch();
   k_di_clear<<<B, 256, 0, s>>>(tail_dead, ex->di_ctr); note_launch();
   k_di_mark_tail<<<B, 256, 0, s>>>(mv, ex->di_ctr, tail_dead, low); note_launch();
   k_di_tail_surv<<<B, 256, 0, s>>>(tail_dead, ex->di_ctr, surv); note_launch();
@@ -561,12 +564,13 @@ int di_remove_holes(vpic_ctx *c, vpic_particle_t *p, const vpic_mover_t *mv, con
 // departures k_move_movers stores into the round r+1 inboxes.  Counts stay
 // on the device; one host synchronisation at the end (the new np).
 int migrate_di(vpic_ctx *c, float qsp, vpic_particle_t *p, int64_t *np_io, int64_t max_np,
-               vpic_mover_t *movers, const int64_t *n_movers, float *acc, cudaStream_t s) {
+               vpic_mover_t *movers, int64_t max_movers, const int64_t *n_movers, float *acc,
+               cudaStream_t s) {
   Exchange *ex = c->ex;
   int32_t *d_flags = reinterpret_cast<int32_t *>(c->d_count + 1);
   CKC(cudaMemsetAsync(d_flags, 0, 4, s));
   k_di_set<<<1, 1, 0, s>>>(ex->di_ctr, *np_io); note_launch();
-  if (int rc = di_remove_holes(c, p, movers, n_movers, s)) return rc;
+  if (int rc = di_remove_holes(c, p, movers, n_movers, max_movers, s)) return rc;
   const int64_t acap = 6 * ex->di_cap;
   const unsigned B = (unsigned)c->num_sms * 4;
   unsigned char *inbox = static_cast<unsigned char *>(ex->di_buf);
@@ -582,7 +586,7 @@ int migrate_di(vpic_ctx *c, float qsp, vpic_particle_t *p, int64_t *np_io, int64
         : launch_move_movers_fast(c, qsp, p, ex->di_arr, acap, acc, ex->di_next, acap, ex->di_ctr + 3,
                                   d_flags, s, ex->di_ctr + 2, r + 1);
     CKC(e);
-    if (int rc = di_remove_holes(c, p, ex->di_next, ex->di_ctr + 3, s)) return rc;
+    if (int rc = di_remove_holes(c, p, ex->di_next, ex->di_ctr + 3, acap, s)) return rc;
   }
   int64_t h_np = 0;
   int32_t h_fl[2] = {0, 0};
@@ -704,12 +708,14 @@ namespace {
 // receives cannot be ambiguous even where one rank is the neighbour in
 // several directions.
 int migrate_ghost(vpic_ctx *c, vpic_particle_t *p, int64_t *np_io, int64_t max_np,
-                  const vpic_mover_t *movers, const int64_t *n_movers, float *acc, cudaStream_t s) {
+                  const vpic_mover_t *movers, int64_t max_movers, const int64_t *n_movers, float *acc,
+                  cudaStream_t s) {
   Exchange *ex = c->ex;
   int64_t M = 0;
   CKC(cudaMemcpyAsync(&M, n_movers, 8, cudaMemcpyDeviceToHost, s));
   CKC(cudaStreamSynchronize(s));
   int64_t np = *np_io;
+  if (M > max_movers) return VPIC_ERR_CAPACITY;   // movers were dropped by advance_p
   if (M > np) return VPIC_ERR_INVALID;
   const int64_t Mpad = std::max<int64_t>(M, 1);
   if (int rc = ctx_scratch(c, 16 * (size_t)Mpad + 64)) return rc;
@@ -783,13 +789,14 @@ int migrate_ghost(vpic_ctx *c, vpic_particle_t *p, int64_t *np_io, int64_t max_n
 // one LSA barrier, append the arrivals, reduce the accumulator ghosts.  One
 // host synchronisation (the new np and the overflow flags).
 int migrate_ghost_di(vpic_ctx *c, vpic_particle_t *p, int64_t *np_io, int64_t max_np,
-                     const vpic_mover_t *movers, const int64_t *n_movers, float *acc, cudaStream_t s) {
+                     const vpic_mover_t *movers, int64_t max_movers, const int64_t *n_movers,
+                     float *acc, cudaStream_t s) {
   Exchange *ex = c->ex;
   const int e = (int)(c->di_epoch & 1);
   int32_t *d_flags = reinterpret_cast<int32_t *>(c->d_count + 1);
   CKC(cudaMemsetAsync(d_flags, 0, 4, s));
   k_di_set<<<1, 1, 0, s>>>(ex->di_ctr, *np_io); note_launch();
-  if (int rc = di_remove_holes(c, p, movers, n_movers, s)) return rc;
+  if (int rc = di_remove_holes(c, p, movers, n_movers, max_movers, s)) return rc;
   unsigned char *inbox = static_cast<unsigned char *>(ex->di_buf);
   k_lsa_barrier<<<1, 128, 0, s>>>(ex->di_dcomm); note_launch();
   k_di_take_ghost<<<1, 32, 0, s>>>(inbox, e, ex->di_cap, max_np, ex->di_ctr, ex->di_flag); note_launch();
@@ -819,15 +826,15 @@ int migrate_ghost_di(vpic_ctx *c, vpic_particle_t *p, int64_t *np_io, int64_t ma
 // CUDA graph and replayed.  The epoch parity is fixed at enqueue time (each
 // call flips it), so a captured sequence must hold an even number of calls.
 int migrate_dev(vpic_ctx *c, vpic_particle_t *p, int64_t *np_dev, int64_t max_np,
-                const vpic_mover_t *movers, const int64_t *n_movers, float *acc, int32_t *flags_dev,
-                cudaStream_t s) {
+                const vpic_mover_t *movers, int64_t max_movers, const int64_t *n_movers, float *acc,
+                int32_t *flags_dev, cudaStream_t s) {
   Exchange *ex = c->ex;
   if (!ex || !ex->di || !c->gk.ghost_mig) return VPIC_ERR_UNSUPPORTED;
   const int e = (int)(c->di_epoch & 1);
   int32_t *d_flags = reinterpret_cast<int32_t *>(c->d_count + 1);
   CKC(cudaMemsetAsync(d_flags, 0, 4, s));
   k_di_set_dev<<<1, 1, 0, s>>>(ex->di_ctr, np_dev); note_launch();
-  if (int rc = di_remove_holes(c, p, movers, n_movers, s)) return rc;
+  if (int rc = di_remove_holes(c, p, movers, n_movers, max_movers, s)) return rc;
   unsigned char *inbox = static_cast<unsigned char *>(ex->di_buf);
   k_lsa_barrier<<<1, 128, 0, s>>>(ex->di_dcomm); note_launch();
   k_di_take_ghost<<<1, 32, 0, s>>>(inbox, e, ex->di_cap, max_np, ex->di_ctr, ex->di_flag); note_launch();
@@ -844,17 +851,20 @@ int migrate_dev(vpic_ctx *c, vpic_particle_t *p, int64_t *np_dev, int64_t max_np
 // Host synchronisations: the initial mover count, one per round (the NCCL
 // record sizes, which also return the round's mover count), one for flags.
 int migrate(vpic_ctx *c, float qsp, float msp, vpic_particle_t *p, int64_t *np_io, int64_t max_np,
-            vpic_mover_t *movers, const int64_t *n_movers, float *acc, cudaStream_t s) {
+            vpic_mover_t *movers, int64_t max_movers, const int64_t *n_movers, float *acc,
+            cudaStream_t s) {
   (void)msp;
   if (c->ex && c->gk.ghost_mig) {
-    return c->ex->di ? migrate_ghost_di(c, p, np_io, max_np, movers, n_movers, acc, s)
-                     : migrate_ghost(c, p, np_io, max_np, movers, n_movers, acc, s);
+    return c->ex->di ? migrate_ghost_di(c, p, np_io, max_np, movers, max_movers, n_movers, acc, s)
+                     : migrate_ghost(c, p, np_io, max_np, movers, max_movers, n_movers, acc, s);
   }
-  if (c->ex && c->ex->di) return migrate_di(c, qsp, p, np_io, max_np, movers, n_movers, acc, s);
+  if (c->ex && c->ex->di)
+    return migrate_di(c, qsp, p, np_io, max_np, movers, max_movers, n_movers, acc, s);
   int64_t M = 0;
   CKC(cudaMemcpyAsync(&M, n_movers, 8, cudaMemcpyDeviceToHost, s));
   CKC(cudaStreamSynchronize(s));
   int64_t np = *np_io;
+  if (M > max_movers) return VPIC_ERR_CAPACITY;   // movers were dropped by advance_p
   if (M > np) return VPIC_ERR_INVALID;
   int32_t *d_flags = reinterpret_cast<int32_t *>(c->d_count + 1);
   CKC(cudaMemsetAsync(d_flags, 0, 4, s));

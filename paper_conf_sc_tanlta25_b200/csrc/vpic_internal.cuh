@@ -179,12 +179,13 @@ cudaError_t launch_sort(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_
                         cudaStream_t s);
 
 int migrate(vpic_ctx *c, float qsp, float msp, vpic_particle_t *p, int64_t *np, int64_t max_np,
-            vpic_mover_t *movers, const int64_t *n_movers, float *acc, cudaStream_t s);
+            vpic_mover_t *movers, int64_t max_movers, const int64_t *n_movers, float *acc,
+            cudaStream_t s);
 // single-round, device-initiated migration with the particle count on the
 // device: no host synchronisation (capturable in a CUDA graph)
 int migrate_dev(vpic_ctx *c, vpic_particle_t *p, int64_t *np_dev, int64_t max_np,
-                const vpic_mover_t *movers, const int64_t *n_movers, float *acc, int32_t *flags_dev,
-                cudaStream_t s);
+                const vpic_mover_t *movers, int64_t max_movers, const int64_t *n_movers, float *acc,
+                int32_t *flags_dev, cudaStream_t s);
 int exchange_create(vpic_ctx *c, const uint8_t *uid);
 void exchange_destroy(vpic_ctx *c);
 // dir = +1: fill the +x/+y/+z ghost planes from the +neighbours' plane 1;

@@ -224,8 +224,12 @@ class HotPath:
                 e1.record(stream)
                 self.adv_events.append((e0, e1, s.np))
             if self.migrate:
+                # VPIC_ERR_CAPACITY (raised) if advance_p dropped movers
                 s.np = vpic.vpic_migrate_particles(self.ctx, s.q, s.m, s.p, s.np, s.p.shape[0],
-                                                   s.movers, s.n_movers, self.acc)
+                                                   s.movers, s.movers.shape[0], s.n_movers, self.acc)
+                fl = int(s.flags.item())      # (the stream is synchronised by the migration)
+                if fl:
+                    raise vpic.VpicError(f"advance_p ({s.name}: flags {fl:#x})", vpic.VPIC_ERR_CAPACITY)
                 s.n_movers.zero_()
         vpic.vpic_unload_accumulator(self.ctx, self.acc, self.jf)
         if self.field_solve:
@@ -263,7 +267,7 @@ class HotPath:
                                     s.movers, s.movers.shape[0], s.n_movers, s.flags)
             if self.migrate:
                 vpic.vpic_migrate_particles_dev(self.ctx, s.q, s.m, s.p, s.np_dev, s.p.shape[0], s.movers,
-                                                s.n_movers, self.acc, s.flags)
+                                                s.movers.shape[0], s.n_movers, self.acc, s.flags)
                 s.n_movers.zero_()
         vpic.vpic_unload_accumulator(self.ctx, self.acc, self.jf)
         if self.field_solve:

@@ -85,9 +85,9 @@ def load(path: str = LIB_PATH) -> ctypes.CDLL:
         "vpic_continuity_residual": ([P, P, P, P, P, P, P], I),
         "vpic_advance_e": ([P, P, P, ctypes.c_float, P], I),
         "vpic_migrate_particles": ([P, ctypes.c_float, ctypes.c_float, P, ctypes.POINTER(I64),
-                                    I64, P, P, P, P], I),
+                                    I64, P, I64, P, P, P], I),
         "vpic_advance_p_dev": ([P, ctypes.c_float, ctypes.c_float, P, P, I64, P, P, P, I64, P, P, P], I),
-        "vpic_migrate_particles_dev": ([P, ctypes.c_float, ctypes.c_float, P, P, I64, P, P, P, P, P], I),
+        "vpic_migrate_particles_dev": ([P, ctypes.c_float, ctypes.c_float, P, P, I64, P, I64, P, P, P, P], I),
     }
     for name, (args, res) in sig.items():
         f = getattr(lib, name)
@@ -243,11 +243,11 @@ def vpic_continuity_residual(ctx: Context, rho0, rho1, jf, out, res=None, stream
 
 
 def vpic_migrate_particles(ctx: Context, q: float, m: float, p, np_: int, max_np: int, movers,
-                           n_movers, acc, stream=None) -> int:
+                           max_movers: int, n_movers, acc, stream=None) -> int:
     n = ctypes.c_int64(np_)
     _check("vpic_migrate_particles", load().vpic_migrate_particles(
-        ctx.h, q, m, _ptr(p), ctypes.byref(n), max_np, _ptr(movers), _ptr(n_movers), _ptr(acc),
-        _stream(stream)))
+        ctx.h, q, m, _ptr(p), ctypes.byref(n), max_np, _ptr(movers), max_movers, _ptr(n_movers),
+        _ptr(acc), _stream(stream)))
     return int(n.value)
 
 
@@ -260,12 +260,12 @@ def vpic_advance_p_dev(ctx: Context, q: float, m: float, p, np_dev, max_np: int,
 
 
 def vpic_migrate_particles_dev(ctx: Context, q: float, m: float, p, np_dev, max_np: int, movers,
-                               n_movers, acc, flags, stream=None):
+                               max_movers: int, n_movers, acc, flags, stream=None):
     """vpic_migrate_particles with the count in device memory: no host
     synchronisation (single-round, device-initiated exchange only)."""
     _check("vpic_migrate_particles_dev", load().vpic_migrate_particles_dev(
-        ctx.h, q, m, _ptr(p), _ptr(np_dev), max_np, _ptr(movers), _ptr(n_movers), _ptr(acc),
-        _ptr(flags), _stream(stream)))
+        ctx.h, q, m, _ptr(p), _ptr(np_dev), max_np, _ptr(movers), max_movers, _ptr(n_movers),
+        _ptr(acc), _ptr(flags), _stream(stream)))
 
 
 # ------------------------------------------------------- tensor helpers --

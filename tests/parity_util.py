@@ -43,16 +43,20 @@ def assert_particles_close(g, gpu, orc, u_old, kick=None):
     d = d - n * np.round(d / n)
     off_err = 2 * np.abs(d)   # offset units: 2 per cell
     assert off_err.max(initial=0) <= OFFSET_TOL, f"max offset err {off_err.max()}"
+    need_kick = np.zeros(gpu.shape[0], bool)
     for k, c in enumerate(("ux", "uy", "uz")):
         ug, uo = gpu[c].astype(np.float64), orc[c].astype(np.float64)
         scale = np.maximum(np.abs(uo), np.abs(u_old[:, k]))
+        base = np.maximum(4 * np.spacing(np.abs(orc[c])).astype(np.float64), 1e-6 * scale)
         if kick is not None:
             scale = np.maximum(scale, kick[:, k])
         tol = np.maximum(4 * np.spacing(np.abs(orc[c])).astype(np.float64), 1e-6 * scale)
         err = np.abs(ug - uo)
+        need_kick |= err > base
         bad = np.nonzero(err > tol)[0]
         assert bad.size == 0, f"{c}: {bad.size} out of tol, worst {err[bad].max()} vs {tol[bad].min()}"
     assert np.array_equal(gpu["w"], orc["w"])
+    return int(need_kick.sum())   # particles within T2 only thanks to its kick term
 
 
 def assert_acc_close(acc_gpu, acc_orc, acc_abs, rel=1e-5):

@@ -223,3 +223,26 @@ def test_graph_mode_matches_eager(V, exchange):
             assert np.array_equal(pa[k].view(np.uint32), pb[k].view(np.uint32))
     vox = g.interior_voxels()
     assert np.abs(ja[vox] - jb[vox]).max() <= 1e-5 * np.abs(ja[vox]).max() * 8
+
+
+@pytest.mark.parametrize("exchange,migration", [("nccl", "rounds"), ("nccl", "single"),
+                                                ("device", "rounds"), ("device", "single")])
+def test_mover_list_overflow_refused(V, exchange, migration):
+    """advance_p with a mover list smaller than the step's departures: the
+    push drops the excess (flags bit 0) and vpic_migrate_particles -- every
+    exchange path -- reports VPIC_ERR_CAPACITY instead of reading movers past
+    the list (migrate took the count from *n_movers unclamped)."""
+    import gc
+    from paper_conf_sc_tanlta25_b200.pic import HotPath
+    gc.collect()
+    g = inputs.GridSpec(6, 5, 4, dt=0.5)
+    wl = inputs.Workload("mv_overflow", g, [inputs.Species("electron", -1.0, 1.0, 0.8)], 60, 1, 0)
+    parts = inputs.make_species_particles(wl)
+    hp = HotPath(wl, parts, inputs.make_fields(g, 0.05), loopback_exchange=True,
+                 device_exchange=exchange == "device", inbox_cap=1 << 16, capacity_factor=1.0,
+                 single_round=migration == "single", max_movers=8)
+    with pytest.raises(V.VpicError) as ei:
+        hp.step()
+    assert ei.value.status == -2      # VPIC_ERR_CAPACITY
+    torch.cuda.synchronize()
+    hp.close()

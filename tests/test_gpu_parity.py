@@ -181,7 +181,7 @@ def run_both(V, orc, g, p, q, m, fields, math, deposit, kernel=0):
     return dict(interp_o=interp_o, acc_o=acc_o, acc_abs=acc_abs, p_o=p_o, mv_o=mv_o,
                 interp=interp.cpu().numpy(), acc=acc.cpu().numpy(), p=V.particles_to_host(pd),
                 nm=int(nm.item()), flags=int(flags.item()), ctx=ctx, fields=fd.cpu().numpy(),
-                acc_t=acc)
+                acc_t=acc, movers=movers.cpu().numpy())
 
 
 @pytest.mark.parametrize("case", adv_cases(), ids=lambda c: c[0])
@@ -203,14 +203,10 @@ def test_advance_ieee_bitexact(V, orc, case, deposit, kernel):
 @pytest.mark.parametrize("kernel", [1, 2], ids=["direct", "tma"])
 def test_advance_fast_tolerance(V, orc, case, deposit, kernel):
     name, g, p, q, m, f = case
-    if name == "scattered_cache_overflow":
-        # ~2 particles per voxel: an entry can hold ONE partial q ux (1 - dy)...
-        # with dy ~ +-1, whose FMA-contracted value differs from the oracle's
-        # by ~ulp(q ux), far above 1e-5 of the cancelled partial (T1 bounds
-        # reordering, not FAST-mode arithmetic); IEEE mode checks this case
-        pytest.skip("IEEE-only case (sparse entries: FAST-mode FMA vs T1)")
     r = run_both(V, orc, g, p, q, m, f, V.MATH_FAST, deposit, kernel)
-    assert_particles_close(g, r["p"], r["p_o"], u_of(p), kick_bound(g, p, q, m, r["interp_o"]))
+    nkick = assert_particles_close(g, r["p"], r["p_o"], u_of(p), kick_bound(g, p, q, m, r["interp_o"]))
+    # T2's kick term is a rare exception, not the working tolerance
+    assert nkick <= max(2, p.size // 2000), nkick
     assert_acc_close(r["acc"], r["acc_o"], r["acc_abs"])
 
 
@@ -277,7 +273,8 @@ def test_absorb_movers_and_migrate(V, orc, kernel):
     # rebuild the mover list on the device from the oracle's (same set)
     movers = torch.from_numpy(r["mv_o"].copy().view(np.float32).reshape(-1, 4)).cuda()
     nm = torch.tensor([r["mv_o"].size], dtype=torch.int64, device="cuda")
-    n_new = V.vpic_migrate_particles(ctx, -1.0, 1.0, pd, p.size, p.size, movers, nm, r["acc_t"])
+    n_new = V.vpic_migrate_particles(ctx, -1.0, 1.0, pd, p.size, p.size, movers, movers.shape[0], nm,
+                                     r["acc_t"])
     p_left_o = orc.remove_absorbed(g, r["p_o"].copy(), r["mv_o"])
     assert n_new == p_left_o.size
     got = V.particles_to_host(pd[:n_new])
@@ -300,6 +297,12 @@ def test_mover_overflow_flag(V, orc):
     V.vpic_advance_p(ctx, -1.0, 1.0, pd, p.size, interp, acc, movers, 4, nm, flags)
     torch.cuda.synchronize()
     assert int(nm.item()) > 4 and int(flags.item()) & 1
+    # the migration refuses the overflowed list before touching anything
+    before = V.particles_to_host(pd)
+    with pytest.raises(V.VpicError) as ei:
+        V.vpic_migrate_particles(ctx, -1.0, 1.0, pd, p.size, p.size, movers, 4, nm, acc)
+    assert ei.value.status == V.VPIC_ERR_CAPACITY
+    assert_particles_bitexact(V.particles_to_host(pd), before)
 
 
 def test_invalid_arguments(V):
@@ -386,3 +389,93 @@ def test_advance_chunk_edges_ieee(V, orc, n, deposit):
     r = run_both(V, orc, g, p, -1.0, 1.0, inputs.make_fields(g, 0.05, seed=8), V.MATH_IEEE, deposit, 2)
     assert_particles_bitexact(r["p"], r["p_o"])
     assert_acc_close(r["acc"], r["acc_o"], r["acc_abs"])
+
+
+# ------------------------------------------ move_p edge cases (reading R13) --
+def edge_case_particles(g):
+    """Particles built so that move_p meets its degenerate branches, with the
+    fields zero (u is unchanged by the push, so the displacements below are
+    exact): on a face moving out of it (zero-length first streak), on a face
+    moving in, zero displacement on one or two axes (the 3.4e38 branch), exact
+    two- and three-face ties (equal offsets and momenta on a cubic grid: the
+    lower axis wins, strict '<'), a track ending exactly on a face (in-cell,
+    d = +-1 kept), and corner crossings through the periodic wrap."""
+    cells = [(x, y, z) for z in (1, 2, g.nz) for y in (1, 2, g.ny) for x in (1, 2, g.nx)]
+    rows = []
+    u = 0.5
+    for s in (+1.0, -1.0):
+        rows += [((s, 0.3, -0.2), (s * u, 0.1, 0.0)),          # on +-x face, moving out
+                 ((0.2, s, 0.1), (0.0, s * u, -0.2)),          # on +-y face, moving out, ux = 0
+                 ((0.1, -0.4, s), (0.0, 0.0, s * u)),          # on +-z face, only z moving
+                 ((s, s, 0.0), (s * u, s * u, 0.0)),           # on an edge, moving out of both
+                 ((s, s, s), (s * u, s * u, s * u)),           # on a corner, moving out of all
+                 ((s, 0.0, 0.0), (-s * u, 0.0, 0.0)),          # on a face, moving in
+                 ((0.9 * s, 0.9 * s, 0.0), (s * u, s * u, 0.0)),       # two-face tie x = y
+                 ((0.0, 0.9 * s, 0.9 * s), (0.0, s * u, s * u)),       # two-face tie y = z
+                 ((0.9 * s, 0.9 * s, 0.9 * s), (s * u, s * u, s * u)),  # three-face tie
+                 ((0.7 * s, -0.7 * s, 0.7 * s), (s * u, -s * u, s * u)),  # three-face tie, mixed signs
+                 ((0.0, 0.0, 0.0), (0.0, 0.0, 0.0)),                  # at rest: all disp == 0
+                 ((0.6 * s, 0.0, 0.0), (2.0 * s, 0.0, 0.0))]          # fast, single axis
+    # a track ending exactly on the face: d + 2 disp == 1 in float32
+    n = len(rows) * len(cells)
+    p = np.zeros(n + len(cells), PD)
+    k = 0
+    for c in cells:
+        for d, uu in rows:
+            p[k]["i"] = g.voxel(*c)
+            p[k]["dx"], p[k]["dy"], p[k]["dz"] = d
+            p[k]["ux"], p[k]["uy"], p[k]["uz"] = uu
+            p[k]["w"] = 0.25 + 0.01 * (k % 7)
+            k += 1
+    # in float32 with VPIC's half displacement (ux c dt / dx) / gamma at ux = 1
+    # (c dt / dx = 0.5 below): the offset whose track ends exactly on +x
+    f32 = np.float32
+    disp = (f32(1.0) * f32(0.5)) * (f32(1.0) / np.sqrt(f32(1.0) + f32(1.0) * f32(1.0)))
+    d_end = f32(1.0) - f32(2.0) * disp
+    for _ in range(8):
+        e = (d_end + disp) + disp
+        if e == f32(1.0):
+            break
+        d_end = np.nextafter(d_end, f32(2.0) if e < 1 else f32(-2.0), dtype=np.float32)
+    assert (d_end + disp) + disp == f32(1.0)
+    for c in cells:
+        p[k]["i"] = g.voxel(*c)
+        p[k]["dx"], p[k]["dy"], p[k]["dz"] = d_end, 0.0, 0.0
+        p[k]["ux"] = 1.0
+        p[k]["w"] = 1.0
+        k += 1
+    return p
+
+
+@pytest.mark.parametrize("pbc", [(0,) * 6, (1, 0, 2, 1, 0, 2)], ids=["periodic", "walls"])
+@pytest.mark.parametrize("deposit", [1, 2, 3], ids=["lane", "warp", "smem"])
+@pytest.mark.parametrize("kernel", [1, 2], ids=["direct", "tma"])
+def test_advance_edge_cases_ieee(V, orc, pbc, deposit, kernel):
+    g = inputs.GridSpec(5, 5, 5, pbc=pbc, dt=0.5)
+    p = edge_case_particles(g)
+    f = np.zeros((g.nv, 8), np.float32)
+    r = run_both(V, orc, g, p, -1.0, 1.0, f, V.MATH_IEEE, deposit, kernel)
+    assert_particles_bitexact(r["p"], r["p_o"])
+    assert_acc_close(r["acc"], r["acc_o"], r["acc_abs"])
+    assert r["nm"] == r["mv_o"].size
+    key = lambda m: np.sort(np.ascontiguousarray(m).view(np.dtype((np.void, 16))))
+    if r["nm"]:
+        # absorbed movers: the same {remaining displacement, index} set
+        mv_gpu = r["movers"][:r["nm"]].copy().view(r["mv_o"].dtype).reshape(-1)
+        assert np.array_equal(key(mv_gpu), key(r["mv_o"]))
+
+
+def test_edge_case_particles_exercise_the_branches(orc):
+    """The edge-case set really reaches the branches it names: crossings with
+    zero-length first streaks, ties, particles left exactly on faces."""
+    g = inputs.GridSpec(5, 5, 5, dt=0.5)
+    p = edge_case_particles(g)
+    f = np.zeros((g.nv, 8), np.float32)
+    interp = orc.load_interpolator(g, f)
+    acc = np.zeros((g.nv, 12), np.float32)
+    p1 = p.copy()
+    orc.advance_p(g, -1.0, 1.0, p1, interp, acc)
+    moved = p1["i"] != p["i"]
+    assert moved.sum() > p.size // 3
+    ended_on_face = p1["dx"][-27:] == 1.0            # the exact end-of-track tie (with 2)
+    assert ended_on_face.all() and np.array_equal(p1["i"][-27:], p["i"][-27:])

@@ -289,3 +289,94 @@ def test_deposit_totals(orc):
         tot = acc[:, 4 * a:4 * a + 4].astype(np.float64).sum()
         exp = 4 * (qw * disp[:, a]).sum()
         assert abs(tot - exp) < 1e-5 * acc_abs[:, 4 * a:4 * a + 4].sum()
+
+
+# ----------------------------------- TV2 / TV3 golden constants (c.5) --
+def _golden():
+    import json
+    import os
+    with open(os.path.join(os.path.dirname(__file__), "golden", "boris_tv2_tv3.json")) as fh:
+        return json.load(fh)
+
+
+def test_tv2_one_step_float32(orc):
+    """TV2: one float32 step of the tan-corrected Boris equals the survey's
+    float32 value (printed to 8 digits: 1 float32 ulp of slack)."""
+    tv = _golden()["TV2_gyration"]
+    g = grid(dt=tv["setup"]["dt"])
+    p = one_particle(g, u=tuple(tv["setup"]["u0"]))
+    us, _ = run(orc, g, p, uniform_fields(g, B=tuple(tv["setup"]["cB"])), 1.0, 1.0, 1, track=True)
+    want = np.array(tv["u_after_one_step_float32"], np.float64)
+    assert np.all(np.abs(us[0] - want) <= np.spacing(np.float32(0.3)).astype(np.float64) * 1.01), (us[0], want)
+
+
+def test_tv2_discrete_rotation_angle_and_radius(orc):
+    """TV2: the discrete rotation per step is theta = 2 atan(v3 |cB|) =
+    0.7241304419859643 (not the continuous 2 phi = 0.72421; a dropped or
+    extra tan-series term moves it by > 1e-5), and the orbit is the regular
+    polygon of circumradius R = 0.3145545360723451 (not r_L = 0.30769)."""
+    tv = _golden()["TV2_gyration"]
+    g = grid(dt=tv["setup"]["dt"])
+    p = one_particle(g, u=tuple(tv["setup"]["u0"]))
+    us, xs = run(orc, g, p, uniform_fields(g, B=tuple(tv["setup"]["cB"])), 1.0, 1.0, 1000, track=True)
+    ang = np.unwrap(np.arctan2(us[:, 1], us[:, 0]))
+    theta = -(ang[-1] - ang[0]) / (len(ang) - 1)
+    assert abs(theta - tv["theta_per_step"]) < 2e-7, theta
+    assert abs(tv["two_phi"] - tv["theta_per_step"]) > 50 * 2e-7   # the pin discriminates
+    a, b, c = xs[:-2, :2], xs[1:-1, :2], xs[2:, :2]
+    la = np.linalg.norm(b - c, axis=1); lb = np.linalg.norm(a - c, axis=1); lc = np.linalg.norm(a - b, axis=1)
+    area = 0.5 * np.abs((b - a)[:, 0] * (c - a)[:, 1] - (b - a)[:, 1] * (c - a)[:, 0])
+    R = np.median(la * lb * lc / (4 * area))
+    assert abs(R - tv["orbit_radius"]) / tv["orbit_radius"] < 1e-4, R
+    assert abs(tv["larmor_radius_continuous"] - tv["orbit_radius"]) / tv["orbit_radius"] > 1e-2
+    assert np.abs(np.linalg.norm(np.diff(xs, axis=0), axis=1) - tv["step_length"]).max() < 2e-6
+
+
+def test_tv3_ExB_discrete_fixed_point(orc):
+    """TV3: with E = (0, 0.01, 0), cB = (0, 0, 1), qdt_2mc = 0.3, the
+    momentum u* = (0.009699099484663786, 0, 0) is a fixed point of the push
+    (to float32 round-off over 1000 steps), while the textbook drift
+    gamma E / cB = 0.0100005 is not (it gyrates about u*)."""
+    tv = _golden()["TV3_ExB_fixed_point"]
+    st = tv["setup"]
+    g = grid(dt=st["dt"])
+    fields = uniform_fields(g, E=tuple(st["E"]), B=tuple(st["cB"]))
+    p = one_particle(g, u=(tv["ux_star"], 0.0, 0.0))
+    us, _ = run(orc, g, p, fields, 1.0, 1.0, 1000, track=True)
+    u0 = np.array([np.float32(tv["ux_star"]), 0.0, 0.0])
+    assert np.abs(us - u0).max() < 2e-8, np.abs(us - u0).max()
+    p = one_particle(g, u=(tv["textbook_gamma_E_over_B"], 0.0, 0.0))
+    us2, _ = run(orc, g, p, fields, 1.0, 1.0, 20, track=True)
+    assert np.abs(us2 - np.array([tv["textbook_gamma_E_over_B"], 0, 0])).max() > 1e-4
+
+
+# ------------------------------------------- orc_remove_absorbed (R12) --
+@pytest.mark.parametrize("seed", [0, 1, 2])
+def test_remove_absorbed_survivors(orc, seed):
+    """Absorbing faces (reading R12): after a push, the particles stopped on
+    an ABSORB face (p.i = 8 voxel + face, pbc[face] == absorb) are removed.
+    Pinned without the oracle's back-fill: the survivors are exactly the
+    multiset of particles NOT listed as absorbed movers, their count is np
+    minus the absorbed ones, particles before the new end that were not
+    removed keep their slot, and movers on a non-absorbing (remote) face
+    are kept."""
+    # absorb on -z/+z, remote (another rank) on +y: both produce movers
+    g = inputs.GridSpec(6, 5, 4, dt=0.5, pbc=(0, 0, 2, 0, 0, 2), nbr_rank=(0, 0, 0, 0, 1, 0))
+    p = inputs.random_particles(g, 4000, 40 + seed, u_scale=1.5)
+    interp = orc.load_interpolator(g, np.zeros((g.nv, 8), np.float32))
+    acc = np.zeros((g.nv, 12), np.float32)
+    mv = orc.advance_p(g, -1.0, 1.0, p, interp, acc)
+    face = p["i"][mv["idx"]] & 7
+    absorbed = np.zeros(p.size, bool)
+    absorbed[mv["idx"][(face == 2) | (face == 5)]] = True
+    remote = mv["idx"][face == 4]
+    assert absorbed.sum() > 50 and remote.size > 50
+    before = p.copy()
+    left = orc.remove_absorbed(g, p, mv)    # the survivors, back-filled in place
+    assert len(left) == before.size - absorbed.sum()
+    key = lambda a: np.sort(np.ascontiguousarray(a).view(np.dtype((np.void, 32))))
+    assert np.array_equal(key(left), key(before[~absorbed]))
+    keep = np.nonzero(~absorbed[:len(left)])[0]
+    assert np.array_equal(left[keep].view(np.uint32), before[keep].view(np.uint32))
+    # remote movers are still there (they leave through migration, not here)
+    assert set(key(before[remote]).tolist()) <= set(key(left).tolist())

@@ -64,9 +64,9 @@ def lib() -> ctypes.CDLL:
         _lib.orc_sort_particles.restype = ctypes.c_int
         _lib.orc_load_interpolator.argtypes = [G, P, P]
         _lib.orc_load_interpolator.restype = None
-        _lib.orc_advance_p.argtypes = [G, ctypes.c_float, ctypes.c_float, P, I64, P, P, P, P, I64]
+        _lib.orc_advance_p.argtypes = [G, ctypes.c_float, ctypes.c_float, P, I64, P, P, P, P, P, I64]
         _lib.orc_advance_p.restype = I64
-        _lib.orc_move_p.argtypes = [G, P, P, P, P, ctypes.c_float]
+        _lib.orc_move_p.argtypes = [G, P, P, P, P, P, ctypes.c_float]
         _lib.orc_move_p.restype = ctypes.c_int
         _lib.orc_unload_accumulator.argtypes = [G, P, P]
         _lib.orc_unload_accumulator.restype = None
@@ -142,8 +142,10 @@ def load_interpolator(spec, fields):
     return interp
 
 
-def advance_p(spec, q, m, p, interp, acc, acc_abs=None, max_movers=None):
-    """In place on p (PARTICLE_DTYPE) and acc (float32[nv,12]). Returns movers."""
+def advance_p(spec, q, m, p, interp, acc, acc_abs=None, max_movers=None, acc_cond=None):
+    """In place on p (PARTICLE_DTYPE) and acc (float32[nv,12]). Returns movers.
+    acc_abs / acc_cond (float64[nv,12], optional): sum of |contribution| and
+    of |q uX| per entry (tolerances T1 / T3)."""
     assert p.dtype == PARTICLE_DTYPE and p.flags.c_contiguous
     assert acc.dtype == np.float32 and acc.flags.c_contiguous
     if max_movers is None:
@@ -151,16 +153,17 @@ def advance_p(spec, q, m, p, interp, acc, acc_abs=None, max_movers=None):
     movers = np.zeros(max(max_movers, 1), MOVER_DTYPE)
     g = make_grid(spec)
     nm = lib().orc_advance_p(ctypes.byref(g), q, m, _ptr(p), p.size, _ptr(interp), _ptr(acc),
-                             _ptr(acc_abs), _ptr(movers), max_movers)
+                             _ptr(acc_abs), _ptr(acc_cond), _ptr(movers), max_movers)
     if nm < 0:
         raise OverflowError("mover list overflow")
     return movers[:nm].copy()
 
 
-def move_p(spec, p1, mover, acc, qsp, acc_abs=None):
+def move_p(spec, p1, mover, acc, qsp, acc_abs=None, acc_cond=None):
     """move_p on a single particle record (np.void / 1-element array) in place."""
     g = make_grid(spec)
-    return lib().orc_move_p(ctypes.byref(g), _ptr(p1), _ptr(mover), _ptr(acc), _ptr(acc_abs), qsp)
+    return lib().orc_move_p(ctypes.byref(g), _ptr(p1), _ptr(mover), _ptr(acc), _ptr(acc_abs),
+                            _ptr(acc_cond), qsp)
 
 
 def unload_accumulator(spec, acc):

@@ -57,17 +57,20 @@ int orc_sort_particles(const orc_grid *g, const orc_particle *in, orc_particle *
 void orc_load_interpolator(const orc_grid *g, float *fields, float *interp);
 
 /* One advance of np particles of species (q, m).  acc[nv][12] is accumulated
- * into; acc_abs (nullable, double[nv][12]) accumulates |contribution|.
+ * into; acc_abs (nullable, double[nv][12]) accumulates |contribution|;
+ * acc_cond (nullable, double[nv][12]) accumulates |q uX| of every streak into
+ * the 4 entries of its component X (test diagnostic: the scale of a partial's
+ * sensitivity to its inputs, for the FAST-mode tolerance T3).
  * Movers (remote/absorb crossings) are appended to movers[]; returns the number
  * appended, or -1 if max_movers was exceeded (excess movers dropped). */
 int64_t orc_advance_p(const orc_grid *g, float q, float m, orc_particle *p, int64_t np,
-                      const float *interp, float *acc, double *acc_abs,
+                      const float *interp, float *acc, double *acc_abs, double *acc_cond,
                       orc_mover *movers, int64_t max_movers);
 
 /* move_p for a single mover (exposed for tests). Returns 1 if the mover is
  * still in use (remote / absorb face reached), else 0. */
 int orc_move_p(const orc_grid *g, orc_particle *p, orc_mover *pm, float *acc,
-               double *acc_abs, float qsp);
+               double *acc_abs, double *acc_cond, float qsp);
 
 /* jf[nv][4] (jfx,jfy,jfz,0) from acc[nv][12]; locally periodic planes folded. */
 void orc_unload_accumulator(const orc_grid *g, const float *acc, float *jf);

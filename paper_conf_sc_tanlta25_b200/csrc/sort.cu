@@ -18,6 +18,13 @@
 // The rank of a particle among equal keys is its stable rank (reading R1), so
 // the result equals Alg. 1/2 with the atomic_fetch_add loop run in input
 // order: keys, counts and permutation are bit-exact against the oracle.
+// Nothing synchronises with the host: the rank passes are launched for the
+// worst case the host can bound (8-bit digits from the least significant;
+// strided keys r < np in 32 bits, tiled keys (chunk - chunk0) max_r + r in 64
+// bits) and every pass above the bits the device finds it needs (max_r, min_k,
+// max_k are device values) returns at once; the record gather picks the
+// buffer the last live pass wrote.  Every order is stream-ordered and can be
+// captured in a CUDA graph.
 #include <algorithm>
 
 #include "vpic_internal.cuh"
@@ -49,7 +56,7 @@ constexpr int TILE = NT * IPT;      // 6144 elements per tile
 // (another box: 512 x 12 x 2 13.84 / 10.48; 384 x 16 x 2 13.84 / 10.48;
 // 512 x 10 x 2 14.40 / 10.99; 1024 x 6 x 1 16.64 / 12.90)
 constexpr int MAX_BITS = 8;         // digit width: 256 buckets, one look-back chain per thread
-constexpr int MAX_PASSES = 4;       // keys up to 32 bits
+constexpr int MAX_PASSES = 8;       // keys up to 64 bits (tiled-strided composite keys)
 constexpr unsigned FULL = 0xffffffffu;
 
 constexpr unsigned long long FLAG_AGG = 1ull << 62;
@@ -233,33 +240,38 @@ __global__ void k_scan_hist(const uint32_t *__restrict__ ghist, uint32_t *__rest
 // ranked, looked back and scattered.  Deadlock-free: a CTA holds at most two
 // tickets, processes them in increasing order, and a tile only waits on
 // smaller tickets, all held by resident CTAs.
-template <int BITS>
+// live_bits (nullable): the pass returns at once (every CTA) when its digit
+// lies above the key width the device found (*live_bits), so the host can
+// launch the worst-case number of passes without reading it back.
+template <int BITS, class KeyT>
 __global__ void __launch_bounds__(NT, VPIC_SORT_MINB)
-k_radix_pass(const uint32_t *__restrict__ kin, const uint32_t *__restrict__ vin,
-             uint32_t *__restrict__ kout, uint32_t *__restrict__ vout, int64_t n, int shift,
+k_radix_pass(const KeyT *__restrict__ kin, const uint32_t *__restrict__ vin,
+             KeyT *__restrict__ kout, uint32_t *__restrict__ vout, int64_t n, int shift,
              const uint32_t *__restrict__ dig_off, unsigned long long *__restrict__ status,
-             unsigned int *__restrict__ tile_ctr) {
+             unsigned int *__restrict__ tile_ctr, const int *__restrict__ live_bits) {
+  if (live_bits && shift > 0 && shift >= *live_bits) return;
   constexpr int NB = 1 << BITS;
   extern __shared__ __align__(16) unsigned char smem[];
   uint16_t *whist = reinterpret_cast<uint16_t *>(smem);                       // [NW][NB]
   uint32_t *tpref = reinterpret_cast<uint32_t *>(smem + NW * NB * 2);          // [NB]
   uint32_t *tstart = tpref + NB;                                               // [NB]
-  uint32_t *skey = tstart + NB;                                                // [TILE]
-  uint32_t *sval = skey + TILE;                                                // [TILE]
+  KeyT *skey = reinterpret_cast<KeyT *>(tstart + NB);                          // [TILE]
+  uint32_t *sval = reinterpret_cast<uint32_t *>(skey + TILE);                  // [TILE]
   __shared__ unsigned int s_tile;
   __shared__ uint32_t wsum[NW];
   const int64_t ntiles = (n + TILE - 1) / TILE;
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const unsigned lt = lanemask_lt();
   uint16_t *wh = whist + w * NB;
-  uint32_t key[IPT], val[IPT];
-  auto load_tile = [&](int64_t t, uint32_t *k, uint32_t *v) {
+  KeyT key[IPT];
+  uint32_t val[IPT];
+  auto load_tile = [&](int64_t t, KeyT *k, uint32_t *v) {
     const int64_t wb = t * TILE + (int64_t)w * 32 * IPT;
 #pragma unroll
     for (int j = 0; j < IPT; ++j) {
       const int64_t i = wb + j * 32 + lane;
       const bool valid = i < n;
-      k[j] = valid ? __ldcs(kin + i) : 0u;
+      k[j] = valid ? __ldcs(kin + i) : KeyT(0);
       v[j] = valid ? (vin ? __ldcs(vin + i) : (uint32_t)i) : 0u;
     }
   };
@@ -285,7 +297,7 @@ k_radix_pass(const uint32_t *__restrict__ kin, const uint32_t *__restrict__ vin,
     for (int j = 0; j < IPT; ++j) {
       const int64_t i = wbase + j * 32 + lane;
       const bool valid = i < n;
-      const uint32_t d = valid ? ((key[j] >> shift) & (NB - 1)) : (uint32_t)NB;
+      const uint32_t d = valid ? (uint32_t)((key[j] >> shift) & (NB - 1)) : (uint32_t)NB;
       const unsigned peers = __match_any_sync(FULL, d);
       uint32_t cur = 0;
       if (valid) cur = wh[d];
@@ -296,7 +308,8 @@ k_radix_pass(const uint32_t *__restrict__ kin, const uint32_t *__restrict__ vin,
       if (j & 1) rank[j >> 1] |= r << 16; else rank[j >> 1] = r;
     }
 #if VPIC_SORT_PERSIST
-    uint32_t nkey[IPT], nval[IPT];
+    KeyT nkey[IPT];
+    uint32_t nval[IPT];
     if (next < ntiles) load_tile(next, nkey, nval);
 #endif
     __syncthreads();
@@ -353,7 +366,7 @@ k_radix_pass(const uint32_t *__restrict__ kin, const uint32_t *__restrict__ vin,
     for (int j = 0; j < IPT; ++j) {
       const int64_t i = wbase + j * 32 + lane;
       if (i < n) {
-        const uint32_t d = (key[j] >> shift) & (NB - 1);
+        const uint32_t d = (uint32_t)((key[j] >> shift) & (NB - 1));
         const uint32_t r = (j & 1) ? (rank[j >> 1] >> 16) : (rank[j >> 1] & 0xffffu);
         const uint32_t lp = tstart[d] + whist[w * NB + d] + r;
         skey[lp] = key[j];
@@ -364,8 +377,8 @@ k_radix_pass(const uint32_t *__restrict__ kin, const uint32_t *__restrict__ vin,
     const int64_t t0 = tile * TILE;
     const int nvalid = (int)(n - t0 < TILE ? n - t0 : (int64_t)TILE);
     for (int e = threadIdx.x; e < nvalid; e += NT) {
-      const uint32_t k = skey[e];
-      const uint32_t d = (k >> shift) & (NB - 1);
+      const KeyT k = skey[e];
+      const uint32_t d = (uint32_t)((k >> shift) & (NB - 1));
       const uint32_t pos = tpref[d] + (uint32_t)e - tstart[d];
       if (kout) kout[pos] = k;
       vout[pos] = sval[e];
@@ -382,14 +395,42 @@ k_radix_pass(const uint32_t *__restrict__ kin, const uint32_t *__restrict__ vin,
   }
 }
 
+// Device-side sizing of the rank passes (no host round trip): from max_r
+// (k_scan_blocksum), min_k = K[0] and max_k = K[n-1] of the standard order.
+struct RankParams {
+  int64_t min_k, max_k, chunk0;
+  uint64_t max_ck;   // largest rank-pass key
+  uint32_t max_r;
+  int nbits;         // bits of max_ck (>= 1): passes with shift >= nbits are skipped
+  int sel;           // the buffer the last live pass writes (number of live passes & 1)
+};
+__global__ void k_rank_setup(const uint32_t *__restrict__ K, int64_t n, int order, int64_t T,
+                             const unsigned int *__restrict__ max_r_dev, RankParams *rp) {
+  RankParams r;
+  r.max_r = *max_r_dev;
+  r.min_k = K[0];
+  r.max_k = K[n - 1];
+  r.chunk0 = r.min_k / T;
+  const uint64_t rmax = r.max_r ? r.max_r - 1 : 0;
+  r.max_ck = order == VPIC_SORT_STRIDED ? rmax
+                                        : (uint64_t)(r.max_k / T - r.chunk0) * r.max_r + rmax;
+  int b = 1;
+  while (b < 64 && (r.max_ck >> b)) ++b;
+  r.nbits = b;
+  const int live = (b + MAX_BITS - 1) / MAX_BITS;
+  r.sel = live & 1;
+  *rp = r;
+}
+
 // Rank-pass keys (strided: r; tiled: (chunk - chunk0) * max_r + r) with the
-// digit histograms of the following passes; optional Alg. 1/2 new keys
-// scattered to the INPUT index (perm_std[j]).
+// digit histograms of the following (worst-case) passes; optional Alg. 1/2
+// new keys scattered to the INPUT index (perm_std[j]).
+template <class KeyT>
 __global__ void __launch_bounds__(256)
 k_rank_keys(const uint32_t *__restrict__ K, const uint32_t *__restrict__ perm_std,
-            const uint32_t *__restrict__ offs, int64_t n, int order, int64_t T, uint32_t max_r,
-            uint32_t *__restrict__ ckey, PassDesc pd, uint32_t *__restrict__ ghist,
-            int64_t *__restrict__ new_keys) {
+            const uint32_t *__restrict__ offs, int64_t n, int order, int64_t T,
+            const RankParams *__restrict__ rp, KeyT *__restrict__ ckey, PassDesc pd,
+            uint32_t *__restrict__ ghist, int64_t *__restrict__ new_keys) {
   extern __shared__ uint32_t sh[];
   int off[MAX_PASSES];
   int tot = 0;
@@ -397,28 +438,30 @@ k_rank_keys(const uint32_t *__restrict__ K, const uint32_t *__restrict__ perm_st
   for (int i = threadIdx.x; i < tot; i += blockDim.x) sh[i] = 0;
   __syncthreads();
   const int lane = threadIdx.x & 31;
-  const int64_t min_k = K[0], max_k = K[n - 1];
-  const int64_t chunk0 = min_k / T;
+  const int64_t min_k = rp->min_k, max_k = rp->max_k, chunk0 = rp->chunk0;
+  const uint64_t max_r = rp->max_r;
+  const int nbits = rp->nbits;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t base = (int64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31); base < n;
        base += stride) {
     const int64_t j = base + lane;
     const bool valid = j < n;
-    uint32_t ck = 0;
+    KeyT ck = 0;
     if (valid) {
       const int64_t k = K[j];
       const int64_t r = j - (int64_t)offs[k];
       if (order == VPIC_SORT_STRIDED) {
-        ck = (uint32_t)r;
+        ck = (KeyT)r;
         if (new_keys) new_keys[perm_std[j]] = (k - min_k) + r * (max_k + 1);
       } else {
-        ck = (uint32_t)((k / T - chunk0) * (int64_t)max_r + r);
+        ck = (KeyT)((uint64_t)(k / T - chunk0) * max_r + (uint64_t)r);
         if (new_keys) new_keys[perm_std[j]] = (k / T) * (T * (int64_t)max_r) + r * T + (k - min_k);
       }
       ckey[j] = ck;
     }
     for (int q = 0; q < pd.npass; ++q) {
-      const uint32_t d = valid ? ((ck >> pd.shift[q]) & ((1u << pd.bits[q]) - 1)) : 0xffffffffu;
+      if (pd.shift[q] > 0 && pd.shift[q] >= nbits) break;   // skipped pass (uniform)
+      const uint32_t d = valid ? (uint32_t)((ck >> pd.shift[q]) & ((1u << pd.bits[q]) - 1)) : 0xffffffffu;
       const unsigned peers = __match_any_sync(FULL, d);
       if (valid && (__ffs(peers) - 1) == lane) atomicAdd(&sh[off[q] + d], __popc(peers));
     }
@@ -439,9 +482,13 @@ k_rank_keys(const uint32_t *__restrict__ K, const uint32_t *__restrict__ perm_st
 // 4: 13.9 / 11.1, 8: 14.0 / 10.8, 16: 13.4 / 11.8)
 constexpr int GATHER_ILP = VPIC_GATHER_ILP;
 
+// perm_alt / sel (nullable): the permutation is in perm_alt instead when
+// sel->sel is 1 (the rank passes' output buffer is known on the device only).
 __global__ void __launch_bounds__(256)
 k_gather(const vpic_particle_t *__restrict__ pin, vpic_particle_t *__restrict__ pout,
-         const uint32_t *__restrict__ perm, int64_t n, int64_t *__restrict__ perm64) {
+         const uint32_t *__restrict__ perm_main, const uint32_t *__restrict__ perm_alt,
+         const RankParams *__restrict__ sel, int64_t n, int64_t *__restrict__ perm64) {
+  const uint32_t *__restrict__ perm = (sel && sel->sel) ? perm_alt : perm_main;
   // two lanes per 32-B record (every warp load / store instruction moves 16
   // whole records: sector-complete, stores fully coalesced); each warp owns
   // blocks of 32 x GATHER_ILP half-records and issues all their loads first
@@ -518,13 +565,16 @@ struct WsLayout {
 
 inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
-WsLayout layout(int64_t np, int64_t nv) {
+// key buffers: u32 voxel keys; 8 B per particle for TILED_STRIDED, whose
+// rank-pass keys (chunk - chunk0) max_r + r can need more than 32 bits
+WsLayout layout(int64_t np, int64_t nv, int order) {
   WsLayout L{};
   size_t o = 0;
   auto take = [&](size_t bytes) { size_t r = o; o = align_up(o + bytes, 256); return r; };
   const int64_t tiles = (np + TILE - 1) / TILE;
-  L.keysA = take(4 * (size_t)np);
-  L.keysB = take(4 * (size_t)np);
+  const size_t kb = order == VPIC_SORT_TILED_STRIDED ? 8 : 4;
+  L.keysA = take(kb * (size_t)np);
+  L.keysB = take(kb * (size_t)np);
   L.valsA = take(4 * (size_t)np);
   L.valsB = take(4 * (size_t)np);
   L.offs = take(4 * (size_t)(nv + 1));
@@ -534,14 +584,14 @@ WsLayout layout(int64_t np, int64_t nv) {
   L.goff = take(4 * (size_t)MAX_PASSES * (1 << MAX_BITS));
   L.status = take(8 * (size_t)std::max<int64_t>(tiles, 1) * (1 << MAX_BITS));
   L.ctr = take(4 * MAX_PASSES);
-  L.misc = take(64);
+  L.misc = take(64 + sizeof(RankParams));
   L.total = o;
   return L;
 }
 
 int bits_for(uint64_t max_value) {  // bits needed to hold values 0..max_value
   int b = 0;
-  while (b < 40 && (max_value >> b)) ++b;
+  while (b < 64 && (max_value >> b)) ++b;
   return std::max(b, 1);
 }
 
@@ -563,15 +613,16 @@ PassDesc make_passes(int nbits) {
   return pd;
 }
 
-template <int BITS>
-cudaError_t radix_pass_bits(const uint32_t *kin, const uint32_t *vin, uint32_t *kout,
-                            uint32_t *vout, int64_t n, int shift, const uint32_t *dig_off,
-                            unsigned long long *status, unsigned int *ctr, cudaStream_t s) {
-  const size_t smem = (size_t)NW * (1 << BITS) * 2 + (size_t)(1 << BITS) * 8 + (size_t)TILE * 8;
+template <int BITS, class KeyT>
+cudaError_t radix_pass_bits(const KeyT *kin, const uint32_t *vin, KeyT *kout, uint32_t *vout,
+                            int64_t n, int shift, const uint32_t *dig_off,
+                            unsigned long long *status, unsigned int *ctr, const int *live_bits,
+                            cudaStream_t s) {
+  const size_t smem = (size_t)NW * (1 << BITS) * 2 + (size_t)(1 << BITS) * 8 + (size_t)TILE * (sizeof(KeyT) + 4);
   const int64_t tiles = (n + TILE - 1) / TILE;
   static std::atomic<uint64_t> configured{0};   // > 48 KB only for large tiles; once per device
   once_per_device(configured, [&] {
-    cudaFuncSetAttribute(k_radix_pass<BITS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(k_radix_pass<BITS, KeyT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   });
   int64_t grid = tiles;
 #if VPIC_SORT_PERSIST
@@ -579,20 +630,21 @@ cudaError_t radix_pass_bits(const uint32_t *kin, const uint32_t *vin, uint32_t *
     int dev = 0, sms = 0, per_sm = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_radix_pass<BITS>, NT, smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_radix_pass<BITS, KeyT>, NT, smem);
     grid = std::min<int64_t>(tiles, (int64_t)sms * std::max(per_sm, 1));
   }
 #endif
-  k_radix_pass<BITS><<<(unsigned)grid, NT, smem, s>>>(kin, vin, kout, vout, n, shift, dig_off,
-                                                       status, ctr); note_launch();
+  k_radix_pass<BITS, KeyT><<<(unsigned)grid, NT, smem, s>>>(kin, vin, kout, vout, n, shift, dig_off,
+                                                             status, ctr, live_bits); note_launch();
   return cudaGetLastError();
 }
 
-cudaError_t radix_pass(int bits, const uint32_t *kin, const uint32_t *vin, uint32_t *kout,
-                       uint32_t *vout, int64_t n, int shift, const uint32_t *dig_off,
-                       unsigned long long *status, unsigned int *ctr, cudaStream_t s) {
+template <class KeyT>
+cudaError_t radix_pass(int bits, const KeyT *kin, const uint32_t *vin, KeyT *kout, uint32_t *vout,
+                       int64_t n, int shift, const uint32_t *dig_off, unsigned long long *status,
+                       unsigned int *ctr, const int *live_bits, cudaStream_t s) {
   switch (bits) {
-#define VPIC_RP(B) case B: return radix_pass_bits<B>(kin, vin, kout, vout, n, shift, dig_off, status, ctr, s);
+#define VPIC_RP(B) case B: return radix_pass_bits<B, KeyT>(kin, vin, kout, vout, n, shift, dig_off, status, ctr, live_bits, s);
     VPIC_RP(1) VPIC_RP(2) VPIC_RP(3) VPIC_RP(4) VPIC_RP(5) VPIC_RP(6) VPIC_RP(7) VPIC_RP(8)
 #undef VPIC_RP
     default: return cudaErrorInvalidValue;
@@ -610,23 +662,27 @@ unsigned grid_cap(int64_t n, int threads, int num_sms, int per_sm) {
 #define CK(x) do { cudaError_t e_ = (x); if (e_ != cudaSuccess) return e_; } while (0)
 
 // Run the LSD passes of `pd` over (keys0, vals0 [nullable = iota]).  Returns
-// pointers to the final keys / vals (inside the workspace).
-cudaError_t lsd_sort(const PassDesc &pd, int64_t n, uint32_t *kA, uint32_t *kB, uint32_t *vA,
+// pointers to the final keys / vals (inside the workspace) when every pass
+// runs; with live_bits, trailing passes may return at once on the device and
+// the vals then end in *v_final (an even number of live passes) or the other
+// buffer (odd; RankParams::sel).
+template <class KeyT>
+cudaError_t lsd_sort(const PassDesc &pd, int64_t n, KeyT *kA, KeyT *kB, uint32_t *vA,
                      uint32_t *vB, const uint32_t *vals0, uint32_t *ghist, uint32_t *goff,
                      unsigned long long *status, unsigned int *ctr, bool need_keys_out,
-                     uint32_t **k_final, uint32_t **v_final, cudaStream_t s) {
+                     const int *live_bits, KeyT **k_final, uint32_t **v_final, cudaStream_t s) {
   CK(cudaMemsetAsync(ctr, 0, 4 * MAX_PASSES, s));
   k_scan_hist<<<pd.npass, 256, 0, s>>>(ghist, goff, pd); note_launch();
   CK(cudaGetLastError());
   const int64_t tiles = (n + TILE - 1) / TILE;
-  uint32_t *kin = kA, *kout = kB;
+  KeyT *kin = kA, *kout = kB;
   const uint32_t *vin = vals0;
   uint32_t *vout = (vals0 == vA) ? vB : vA;
   for (int q = 0; q < pd.npass; ++q) {
     CK(cudaMemsetAsync(status, 0, 8 * (size_t)tiles * (1 << pd.bits[q]), s));
     const bool last = q == pd.npass - 1;
-    CK(radix_pass(pd.bits[q], kin, vin, (last && !need_keys_out) ? nullptr : kout, vout, n,
-                  pd.shift[q], goff + q * (1 << MAX_BITS), status, ctr + q, s));
+    CK(radix_pass<KeyT>(pd.bits[q], kin, vin, (last && !need_keys_out) ? nullptr : kout, vout, n,
+                        pd.shift[q], goff + q * (1 << MAX_BITS), status, ctr + q, live_bits, s));
     *k_final = kout;
     *v_final = vout;
     std::swap(kin, kout);
@@ -636,11 +692,54 @@ cudaError_t lsd_sort(const PassDesc &pd, int64_t n, uint32_t *kA, uint32_t *kB, 
   return cudaSuccess;
 }
 
+// Worst-case rank passes: 8-bit digits from the least significant bit.
+PassDesc rank_passes(int nbits) {
+  PassDesc pd{};
+  pd.npass = std::min(MAX_PASSES, std::max(1, (nbits + MAX_BITS - 1) / MAX_BITS));
+  for (int q = 0; q < pd.npass; ++q) {
+    pd.bits[q] = MAX_BITS;
+    pd.shift[q] = MAX_BITS * q;
+  }
+  return pd;
+}
+
+// The rank stage of STRIDED / TILED_STRIDED: keys from the standard order
+// (K, P), passes sized on the device; returns the two candidate perm buffers
+// (the first when the number of live passes is even).
+template <class KeyT>
+cudaError_t rank_stage(vpic_ctx *c, int64_t np, int order, int64_t T, int worst_bits,
+                       const uint32_t *K, uint32_t *P, KeyT *ckA, KeyT *ckB, uint32_t *vfree,
+                       const uint32_t *offs, const unsigned int *max_r_dev, RankParams *rp,
+                       uint32_t *ghist, uint32_t *goff, unsigned long long *status,
+                       unsigned int *ctr, int64_t *new_keys, uint32_t **perm_even,
+                       uint32_t **perm_odd, cudaStream_t s) {
+  k_rank_setup<<<1, 1, 0, s>>>(K, np, order, T, max_r_dev, rp); note_launch();
+  CK(cudaGetLastError());
+  const PassDesc pr = rank_passes(worst_bits);
+  CK(cudaMemsetAsync(ghist, 0, 4 * (size_t)MAX_PASSES * (1 << MAX_BITS), s));
+  int tot = 0;
+  for (int q = 0; q < pr.npass; ++q) tot += 1 << pr.bits[q];
+  static std::atomic<uint64_t> configured{0};
+  once_per_device(configured, [] {
+    cudaFuncSetAttribute(k_rank_keys<KeyT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         4 * MAX_PASSES * (1 << MAX_BITS));
+  });
+  k_rank_keys<KeyT><<<grid_cap(np, 256, c->num_sms, 2), 256, 4 * (size_t)tot, s>>>(
+      K, P, offs, np, order, T, rp, ckA, pr, ghist, new_keys); note_launch();
+  CK(cudaGetLastError());
+  KeyT *kf = nullptr;
+  uint32_t *vf = nullptr;
+  CK(lsd_sort<KeyT>(pr, np, ckA, ckB, P, vfree, P, ghist, goff, status, ctr, false, &rp->nbits,
+                    &kf, &vf, s));
+  *perm_even = P;       // live passes: 2, 4, ...
+  *perm_odd = vfree;    //              1, 3, ...
+  return cudaSuccess;
+}
+
 }  // namespace
 
 size_t sort_workspace_bytes(const vpic_ctx *c, int64_t np, int order) {
-  (void)order;
-  return layout(np, c->gk.nv).total;
+  return layout(np, c->gk.nv, order).total;
 }
 
 cudaError_t launch_sort(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_t *p_out,
@@ -665,7 +764,7 @@ cudaError_t launch_sort(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_
     }
     return cudaSuccess;
   }
-  const WsLayout L = layout(np, nv);
+  const WsLayout L = layout(np, nv, order);
   if (ws_bytes < L.total) return cudaErrorInvalidValue;
   char *w = static_cast<char *>(ws);
   uint32_t *kA = reinterpret_cast<uint32_t *>(w + L.keysA);
@@ -678,6 +777,7 @@ cudaError_t launch_sort(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_
   unsigned long long *status = reinterpret_cast<unsigned long long *>(w + L.status);
   unsigned int *ctr = reinterpret_cast<unsigned int *>(w + L.ctr);
   unsigned int *misc = reinterpret_cast<unsigned int *>(w + L.misc);
+  RankParams *rp = reinterpret_cast<RankParams *>(w + L.misc + 64);
 
   // ---- voxel histogram (deterministic run counts), digit histograms
   uint32_t *count = voxel_counts ? reinterpret_cast<uint32_t *>(voxel_counts)
@@ -693,7 +793,10 @@ cudaError_t launch_sort(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_
   // ---- standard order: stable LSD radix sort of (voxel, index)
   uint32_t *K = nullptr, *P = nullptr;
   const bool need_offs = order != VPIC_SORT_STANDARD;
-  CK(lsd_sort(pd, np, kA, kB, vA, vB, nullptr, ghist, goff, status, ctr, need_offs, &K, &P, s));
+  CK(lsd_sort<uint32_t>(pd, np, kA, kB, vA, vB, nullptr, ghist, goff, status, ctr, need_offs,
+                        nullptr, &K, &P, s));
+  const RankParams *sel = nullptr;
+  uint32_t *P_alt = nullptr;
   if (need_offs) {  // offs[k] = first standard position of voxel k; max_r
     uint32_t *bsum = reinterpret_cast<uint32_t *>(w + L.bsum);
     const int64_t nb = (nv + SCAN_B - 1) / SCAN_B;
@@ -702,45 +805,29 @@ cudaError_t launch_sort(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_
     k_scan_bsums<<<1, 1024, 0, s>>>(bsum, nb); note_launch();
     k_scan_apply<<<(unsigned)nb, 256, 0, s>>>(count, nv, bsum, offs, np); note_launch();
     CK(cudaGetLastError());
-  }
-  if (order == VPIC_SORT_STRIDED || order == VPIC_SORT_TILED_STRIDED) {
-    // host needs max_r, min_k and max_k to size the rank pass (one sync)
-    uint32_t h[3];
-    CK(cudaMemcpyAsync(&h[0], misc, 4, cudaMemcpyDeviceToHost, s));
-    CK(cudaMemcpyAsync(&h[1], K, 4, cudaMemcpyDeviceToHost, s));
-    CK(cudaMemcpyAsync(&h[2], K + np - 1, 4, cudaMemcpyDeviceToHost, s));
-    CK(cudaStreamSynchronize(s));
-    const uint32_t max_r = h[0];
-    const int64_t min_k = h[1], max_k = h[2];
     const int64_t T = tile_sz > 0 ? tile_sz : c->tile_sz;
-    uint64_t max_ck;
-    if (order == VPIC_SORT_STRIDED) max_ck = max_r ? max_r - 1 : 0;
-    else max_ck = (uint64_t)(max_k / T - min_k / T) * max_r + (max_r ? max_r - 1 : 0);
-    if (max_ck >> 32) return cudaErrorInvalidValue;  // composite key beyond 32 bits
-    const PassDesc pr = make_passes(bits_for(max_ck));
-    // the standard keys/perm live in (K, P); use the other buffers for the rank pass
+    // the standard keys/perm live in (K, P); the rank passes use the other
+    // buffers (and K's once the rank keys are written)
     uint32_t *ck = (K == kA) ? kB : kA;
     uint32_t *vfree = (P == vA) ? vB : vA;
-    CK(cudaMemsetAsync(ghist, 0, 4 * (size_t)MAX_PASSES * (1 << MAX_BITS), s));
-    {
-      int tot = 0;
-      for (int q = 0; q < pr.npass; ++q) tot += 1 << pr.bits[q];
-      static std::atomic<uint64_t> configured{0};
-      once_per_device(configured, [] {
-        cudaFuncSetAttribute(k_rank_keys, cudaFuncAttributeMaxDynamicSharedMemorySize, 4 * MAX_PASSES * (1 << MAX_BITS));
-      });
-      k_rank_keys<<<grid_cap(np, 256, sms, 2), 256, 4 * (size_t)tot, s>>>(
-          K, P, offs, np, order, T, max_r, ck, pr, ghist, new_keys); note_launch();
-      CK(cudaGetLastError());
+    uint32_t *Pe = nullptr, *Po = nullptr;
+    if (order == VPIC_SORT_STRIDED) {
+      // r < max_r <= np < 2^32
+      CK(rank_stage<uint32_t>(c, np, order, T, bits_for((uint64_t)(np - 1)), K, P, ck, K, vfree,
+                              offs, misc, rp, ghist, goff, status, ctr, new_keys, &Pe, &Po, s));
+    } else {
+      // (chunk - chunk0) max_r + r <= ((nv - 1) / T) np + np - 1, in 64 bits
+      const uint64_t worst = (uint64_t)((nv - 1) / T) * (uint64_t)np + (uint64_t)(np - 1);
+      CK(rank_stage<uint64_t>(c, np, order, T, bits_for(worst), K, P,
+                              reinterpret_cast<uint64_t *>(ck), reinterpret_cast<uint64_t *>(K), vfree,
+                              offs, misc, rp, ghist, goff, status, ctr, new_keys, &Pe, &Po, s));
     }
-    // the rank pass permutes the standard perm P; K (standard keys) is free now
-    // buffers: keys ck -> other = K ; vals P -> vfree
-    uint32_t *kX = ck, *kY = K, *vX = P, *vY = vfree;
-    uint32_t *K2 = nullptr, *P2 = nullptr;
-    CK(lsd_sort(pr, np, kX, kY, vX, vY, P, ghist, goff, status, ctr, false, &K2, &P2, s));
-    P = P2;
+    P = Pe;
+    P_alt = Po;
+    sel = rp;
   }
-  k_gather<<<grid_cap(2 * np / GATHER_ILP + 1, 256, sms, 8), 256, 0, s>>>(p_in, p_out, P, np, perm); note_launch();
+  k_gather<<<grid_cap(2 * np / GATHER_ILP + 1, 256, sms, 8), 256, 0, s>>>(p_in, p_out, P, P_alt, sel, np,
+                                                                          perm); note_launch();
   return cudaGetLastError();
 }
 

@@ -59,12 +59,18 @@ def assert_particles_close(g, gpu, orc, u_old, kick=None):
     return int(need_kick.sum())   # particles within T2 only thanks to its kick term
 
 
-def assert_acc_close(acc_gpu, acc_orc, acc_abs, rel=1e-5):
-    """|a_gpu - a_orc| <= rel * sum|contributions| per entry (atomic reordering only)."""
+def assert_acc_close(acc_gpu, acc_orc, acc_abs, rel=1e-5, cond=None):
+    """T1: |a_gpu - a_orc| <= rel * sum|contributions| per entry (atomic
+    reordering only: the partials are equal because the streaks are).
+    T3 (FAST mode, cond = the oracle's sum of |q uX| per entry): + rel * cond,
+    the bound of T2's particle tolerance propagated through ACCUMULATE_J
+    (T3).  Returns the number of entries that needed the T3 term."""
     err = np.abs(acc_gpu.astype(np.float64) - acc_orc.astype(np.float64))
-    tol = rel * acc_abs + 1e-30
+    t1 = rel * acc_abs + 1e-30
+    tol = t1 if cond is None else t1 + rel * cond
     bad = np.argwhere(err > tol)
     assert bad.size == 0, f"{len(bad)} acc entries out of tol; worst err {err.max()}, at {bad[:3]}"
+    return int((err > t1).sum())
 
 
 def u_of(p):

@@ -164,8 +164,9 @@ def run_both(V, orc, g, p, q, m, fields, math, deposit, kernel=0):
     interp_o = orc.load_interpolator(g, fields.copy())
     acc_o = np.zeros((g.nv, 12), np.float32)
     acc_abs = np.zeros((g.nv, 12), np.float64)
+    acc_cond = np.zeros((g.nv, 12), np.float64)
     p_o = p.copy()
-    mv_o = orc.advance_p(g, q, m, p_o, interp_o, acc_o, acc_abs)
+    mv_o = orc.advance_p(g, q, m, p_o, interp_o, acc_o, acc_abs, acc_cond=acc_cond)
     ctx = mkctx(V, g, math, deposit, kernel)
     fd = torch.from_numpy(fields.copy()).cuda()
     interp = torch.zeros((g.nv, 24), dtype=torch.float32, device="cuda")
@@ -178,7 +179,7 @@ def run_both(V, orc, g, p, q, m, fields, math, deposit, kernel=0):
     flags = torch.zeros(1, dtype=torch.int32, device="cuda")
     V.vpic_advance_p(ctx, q, m, pd, p.size, interp, acc, movers, p.size, nm, flags)
     torch.cuda.synchronize()
-    return dict(interp_o=interp_o, acc_o=acc_o, acc_abs=acc_abs, p_o=p_o, mv_o=mv_o,
+    return dict(interp_o=interp_o, acc_o=acc_o, acc_abs=acc_abs, acc_cond=acc_cond, p_o=p_o, mv_o=mv_o,
                 interp=interp.cpu().numpy(), acc=acc.cpu().numpy(), p=V.particles_to_host(pd),
                 nm=int(nm.item()), flags=int(flags.item()), ctx=ctx, fields=fd.cpu().numpy(),
                 acc_t=acc, movers=movers.cpu().numpy())
@@ -207,7 +208,12 @@ def test_advance_fast_tolerance(V, orc, case, deposit, kernel):
     nkick = assert_particles_close(g, r["p"], r["p_o"], u_of(p), kick_bound(g, p, q, m, r["interp_o"]))
     # T2's kick term is a rare exception, not the working tolerance
     assert nkick <= max(2, p.size // 2000), nkick
-    assert_acc_close(r["acc"], r["acc_o"], r["acc_abs"])
+    # T3: T1 plus T2 propagated through ACCUMULATE_J; also rare (entries
+    # whose partials cancel: (1 +- dY)(1 +- dZ) ~ 0 with no other contributor)
+    nt3 = assert_acc_close(r["acc"], r["acc_o"], r["acc_abs"], cond=r["acc_cond"])
+    nz = int((r["acc_abs"] > 0).sum())
+    assert nt3 <= max(4, nz // 1000), (nt3, nz)
+    print(f"[{name}] T2 kick term: {nkick} of {p.size} particles; T3 term: {nt3} of {nz} entries")
 
 
 def test_ghost_fill_matches(V, orc):
@@ -479,3 +485,41 @@ def test_edge_case_particles_exercise_the_branches(orc):
     assert moved.sum() > p.size // 3
     ended_on_face = p1["dx"][-27:] == 1.0            # the exact end-of-track tie (with 2)
     assert ended_on_face.all() and np.array_equal(p1["i"][-27:], p["i"][-27:])
+
+
+@pytest.mark.parametrize("order", [0, 1, 2], ids=["standard", "strided", "tiled"])
+def test_sort_captures_in_cuda_graph(V, orc, order):
+    """Every order is stream-ordered with no host synchronisation (the rank
+    passes are sized on the device), so vpic_sort_particles can be captured
+    in a CUDA graph; replays on new input bytes stay bit-exact."""
+    g = inputs.GridSpec(20, 18, 16)
+    ctx = mkctx(V, g)
+    T = 37
+    n = 60001
+    p_in = torch.empty((n, 8), dtype=torch.float32, device="cuda")
+    p_out = torch.empty_like(p_in)
+    ws = torch.empty(V.vpic_sort_workspace_bytes(ctx, n, order), dtype=torch.uint8, device="cuda")
+    counts = torch.empty(g.nv, dtype=torch.int32, device="cuda")
+    nk = torch.empty(n, dtype=torch.int64, device="cuda")
+    perm = torch.empty(n, dtype=torch.int64, device="cuda")
+    p0 = inputs.shuffle(inputs.random_particles(g, n, 71), 72)
+    p_in.copy_(V.particles_to_device(p0))
+    V.vpic_sort_particles(ctx, p_in, p_out, n, order, T, ws, counts, nk, perm)   # warm-up (attributes)
+    torch.cuda.synchronize()
+    s = torch.cuda.Stream()
+    gr = torch.cuda.CUDAGraph()
+    with torch.cuda.stream(s):
+        with torch.cuda.graph(gr, stream=s):
+            V.vpic_sort_particles(ctx, p_in, p_out, n, order, T, ws, counts, nk, perm, stream=s)
+    for seed in (73, 74):
+        # a different key distribution each replay: max_r, min_k, max_k change
+        vox = None if seed == 73 else [g.voxel(3, 4, 5), g.voxel(20, 18, 16), g.voxel(7, 1, 2)]
+        p = inputs.shuffle(inputs.random_particles(g, n, seed, vox=vox), seed + 10)
+        p_in.copy_(V.particles_to_device(p))
+        gr.replay()
+        torch.cuda.synchronize()
+        p_o, c_o, nk_o, perm_o = orc.sort_particles(g, p, order, T)
+        assert_particles_bitexact(V.particles_to_host(p_out), p_o)
+        assert np.array_equal(counts.cpu().numpy(), c_o)
+        assert np.array_equal(nk.cpu().numpy(), nk_o)
+        assert np.array_equal(perm.cpu().numpy(), perm_o)

@@ -66,6 +66,8 @@ def lib() -> ctypes.CDLL:
         _lib.orc_load_interpolator.restype = None
         _lib.orc_advance_p.argtypes = [G, ctypes.c_float, ctypes.c_float, P, I64, P, P, P, P, P, I64]
         _lib.orc_advance_p.restype = I64
+        _lib.orc_move_deposit.argtypes = [G, ctypes.c_float, P, I64, P, P, P, P, I64]
+        _lib.orc_move_deposit.restype = I64
         _lib.orc_move_p.argtypes = [G, P, P, P, P, P, ctypes.c_float]
         _lib.orc_move_p.restype = ctypes.c_int
         _lib.orc_unload_accumulator.argtypes = [G, P, P]
@@ -154,6 +156,22 @@ def advance_p(spec, q, m, p, interp, acc, acc_abs=None, max_movers=None, acc_con
     g = make_grid(spec)
     nm = lib().orc_advance_p(ctypes.byref(g), q, m, _ptr(p), p.size, _ptr(interp), _ptr(acc),
                              _ptr(acc_abs), _ptr(acc_cond), _ptr(movers), max_movers)
+    if nm < 0:
+        raise OverflowError("mover list overflow")
+    return movers[:nm].copy()
+
+
+def move_deposit(spec, q, p, acc, acc_abs=None, max_movers=None):
+    """The move + deposit half of advance_p on particles whose momenta are
+    already pushed (in place on p and acc).  Returns movers."""
+    assert p.dtype == PARTICLE_DTYPE and p.flags.c_contiguous
+    assert acc.dtype == np.float32 and acc.flags.c_contiguous
+    if max_movers is None:
+        max_movers = p.size
+    movers = np.zeros(max(max_movers, 1), MOVER_DTYPE)
+    g = make_grid(spec)
+    nm = lib().orc_move_deposit(ctypes.byref(g), q, _ptr(p), p.size, _ptr(acc), _ptr(acc_abs), None,
+                                _ptr(movers), max_movers)
     if nm < 0:
         raise OverflowError("mover list overflow")
     return movers[:nm].copy()

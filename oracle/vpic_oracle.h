@@ -67,6 +67,12 @@ int64_t orc_advance_p(const orc_grid *g, float q, float m, orc_particle *p, int6
                       const float *interp, float *acc, double *acc_abs, double *acc_cond,
                       orc_mover *movers, int64_t max_movers);
 
+/* The move-and-deposit half of orc_advance_p alone: p[].u must already be
+ * the pushed momentum (replay of another implementation's momenta). */
+int64_t orc_move_deposit(const orc_grid *g, float qsp, orc_particle *p, int64_t np, float *acc,
+                         double *acc_abs, double *acc_cond, orc_mover *movers,
+                         int64_t max_movers);
+
 /* move_p for a single mover (exposed for tests). Returns 1 if the mover is
  * still in use (remote / absorb face reached), else 0. */
 int orc_move_p(const orc_grid *g, orc_particle *p, orc_mover *pm, float *acc,

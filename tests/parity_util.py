@@ -75,3 +75,32 @@ def assert_acc_close(acc_gpu, acc_orc, acc_abs, rel=1e-5, cond=None):
 
 def u_of(p):
     return np.stack([p["ux"], p["uy"], p["uz"]], 1).astype(np.float64)
+
+
+def replay_inputs(orc, g, q, p, p_gpu):
+    """The particles with the GPU's PUSHED momenta (before the move): its
+    final momenta, with the components a reflecting wall negated during the
+    move negated back -- for each particle the one sign pattern (over the
+    reflecting axes) whose oracle move ends in the GPU's final momentum and
+    position."""
+    refl = [a for a in range(3) if g.pbc[a] == inputs.BC_REFLECT or g.pbc[a + 3] == inputs.BC_REFLECT]
+    comps = ("ux", "uy", "uz")
+    chosen = np.full(p.size, -1)
+    pr = p.copy()
+    for c in comps:
+        pr[c] = p_gpu[c]
+    for pat in range(1 << len(refl)):
+        cand = pr.copy()
+        for b, a in enumerate(refl):
+            if pat >> b & 1:
+                cand[comps[a]] = -cand[comps[a]]
+        out = cand.copy()
+        orc.move_deposit(g, q, out, np.zeros((g.nv, 12), np.float32))
+        ok = (out.view(np.uint32).reshape(-1, 8) == p_gpu.view(np.uint32).reshape(-1, 8)).all(1)
+        pick = ok & (chosen < 0)
+        chosen[pick] = pat
+        if pat:
+            for c in comps:
+                pr[c][pick] = cand[c][pick]
+    assert (chosen >= 0).all(), f"{(chosen < 0).sum()} GPU particles are no oracle move of any pushed momentum"
+    return pr

@@ -380,3 +380,22 @@ def test_remove_absorbed_survivors(orc, seed):
     assert np.array_equal(left[keep].view(np.uint32), before[keep].view(np.uint32))
     # remote movers are still there (they leave through migration, not here)
     assert set(key(before[remote]).tolist()) <= set(key(left).tolist())
+
+
+def test_move_deposit_replays_advance(orc):
+    """orc_move_deposit (the replay tool of the FAST-mode parity tests) given
+    the oracle's own pushed momenta reproduces orc_advance_p exactly."""
+    g = inputs.GridSpec(6, 5, 4, dt=0.5, pbc=(0, 0, 2, 0, 0, 1))
+    p = inputs.random_particles(g, 3000, 17, u_scale=1.2)
+    interp = orc.load_interpolator(g, (np.random.default_rng(2).random((g.nv, 8), np.float32) - 0.5) * 0.2)
+    acc = np.zeros((g.nv, 12), np.float32)
+    p1 = p.copy()
+    mv = orc.advance_p(g, -1.0, 1.0, p1, interp, acc)
+    from parity_util import replay_inputs
+    pr = replay_inputs(orc, g, -1.0, p, p1)     # the pushed momenta (reflections undone)
+    assert (pr["uz"] != p1["uz"]).sum() > 0      # some particles were reflected
+    acc_r = np.zeros_like(acc)
+    mv_r = orc.move_deposit(g, -1.0, pr, acc_r)
+    assert np.array_equal(pr.view(np.uint32), p1.view(np.uint32))
+    assert np.array_equal(acc_r.view(np.uint32), acc.view(np.uint32))
+    assert np.array_equal(mv_r.view(np.uint32), mv.view(np.uint32)) and mv.size > 0

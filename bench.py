@@ -42,9 +42,16 @@ def parse():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", type=int, default=1)
-    ap.add_argument("--order", default="standard", choices=["standard", "strided", "tiled_strided", "none"])
-    ap.add_argument("--shuffle", action="store_true", help="random initial order (paper's 'random')")
+    ap.add_argument("--config", type=int, default=1,
+                    help="BASELINE.json configs[] index (0-4); 5 = SURVEY §8(f) f3: L2-resident strong "
+                         "scaling, 256x128x128 uniform, 32 ppc, random order, sorting off")
+    ap.add_argument("--block-of", type=int, default=1,
+                    help="1 GPU: run rank 0's block of the config's box split over this many ranks "
+                         "(locally periodic; the compute side of a strong-scaling point)")
+    ap.add_argument("--order", default=None, choices=["standard", "strided", "tiled_strided", "none"],
+                    help="sort order (default: standard; none for --config 5)")
+    ap.add_argument("--shuffle", action="store_true", help="random initial order (paper's 'random'; "
+                                                           "default for --config 5)")
     ap.add_argument("--sort-every", type=int, default=0)
     ap.add_argument("--math", default="fast", choices=["fast", "ieee"])
     ap.add_argument("--deposit", default="auto", choices=["auto", "lane", "warp", "smem"])
@@ -64,7 +71,12 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no e2e/cpu legs)")
-    return ap.parse_args()
+    a = ap.parse_args()
+    if a.order is None:
+        a.order = "none" if a.config == 5 else "standard"
+    if a.config == 5:
+        a.shuffle = True
+    return a
 
 
 ORDERS = {"standard": 0, "strided": 1, "tiled_strided": 2, "none": 3}
@@ -152,11 +164,34 @@ def oracle_sample_workload(cfg: int = 1):
     from dataclasses import replace
     wl = inputs.config(3 if cfg == 3 else cfg)
     n = {"uniform": (32, 32, 16), "harris": (32, 16, 32), "lpi": (64, 16, 16)}[wl.kind]
+    if cfg == 5:
+        n = (64, 32, 32)
     return replace(wl, grid=replace(wl.grid, nx=n[0], ny=n[1], nz=n[2]),
                    name=wl.name + "@%dx%dx%d" % n)
 
 
-def run_oracle_steps(wl, n_steps, sort_every, order):
+def host_cores() -> int:
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:  # pragma: no cover
+        return os.cpu_count() or 1
+
+
+def cpu_model() -> str:
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            if line.lower().startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return "unknown"
+
+
+def run_oracle_steps(wl, n_steps, sort_every, order, threads=1):
+    """The oracle on the host: per step one sort of each species (serial)
+    and sort_every PIC steps; the push on `threads` cores (orc_advance_p_omp:
+    particle blocks with private accumulators) when threads > 1."""
     import oracle
     from paper_conf_sc_tanlta25_b200 import inputs
     oracle.build()
@@ -174,17 +209,24 @@ def run_oracle_steps(wl, n_steps, sort_every, order):
             interp = oracle.load_interpolator(g, fields)
             acc[:] = 0
             for sp, p in zip(wl.species, parts):
-                oracle.advance_p(g, sp.q, sp.m, p, interp, acc)
+                if threads > 1:
+                    oracle.advance_p_omp(g, sp.q, sp.m, p, interp, acc, threads)
+                else:
+                    oracle.advance_p(g, sp.q, sp.m, p, interp, acc)
                 pushes += p.size
             oracle.unload_accumulator(g, acc)
         times.append(time.perf_counter() - t0)
     return times, sum(p.size for p in parts) * sort_every
 
 
+STRONG_CONFIGS = (4, 5)
+
+
 def effective_config(args, world):
     """The configs[] index a run measures: as given on one GPU; under torchrun
-    the weak-scaling configs[3], or configs[4] split over the ranks (strong)."""
-    return args.config if (world == 1 or args.config == 4) else 3
+    the weak-scaling configs[3], or configs[4] / the f3 box split over the
+    ranks (strong)."""
+    return args.config if (world == 1 or args.config in STRONG_CONFIGS) else 3
 
 
 def reference_arm(args, rank, world):
@@ -195,33 +237,46 @@ def reference_arm(args, rank, world):
     wl = oracle_sample_workload(cfg)
     S = args.sort_every or wl.sort_every
     order = ORDERS[args.order]
-    _ = run_oracle_steps(wl, max(args.warmup, 0) and 1, S, order)  # untimed warm-up (1 step)
-    times, per_step = run_oracle_steps(wl, args.steps, S, order)
+    cores = host_cores()
+    _ = run_oracle_steps(wl, max(args.warmup, 0) and 1, S, order, cores)  # untimed warm-up (1 step)
+    times, per_step = run_oracle_steps(wl, args.steps, S, order, cores)
     total = sum(times)
     value = per_step * args.steps / total
     out = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * total / args.steps,
-        "higher_is_better": True, "scaling": "strong" if (world > 1 and cfg == 4) else "weak",
+        "higher_is_better": True, "scaling": "strong" if (world > 1 and cfg in STRONG_CONFIGS) else "weak",
         "vs_baseline": None, "dtype": "f32",
         "data": "synthetic",
         "config": {"workload": inputs.config(cfg).name, "order": args.order, "sort_every": S,
                    "sample": f"{wl.name}: {per_step // S} particles per step (bounded CPU sample)"},
-        "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
-                         "sample": f"serial C++ oracle (oracle/), {wl.name}: {per_step // S} particles, "
-                                   f"sort + {S} PIC steps per step"},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
+                         "cpu_model": cpu_model(),
+                         "sample": f"C++ oracle (oracle/; push on {cores} cores with OpenMP particle blocks "
+                                   f"and private accumulators, sort serial), {wl.name}: {per_step // S} "
+                                   f"particles, sort + {S} PIC steps per step"},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(out), flush=True)
 
 
 def cpu_baseline(args):
+    """The oracle on this box's host cores (SURVEY.md §8(d) "Oracle timing"):
+    (ii) all cores of the affinity mask (OpenMP particle blocks, private
+    accumulators) -- the reported value -- and (i) one core, serial."""
     wl = oracle_sample_workload(args.config)
     S = args.sort_every or wl.sort_every
-    times, per_step = run_oracle_steps(wl, 1, S, ORDERS[args.order])
-    return {"value": per_step / times[0], "unit": UNIT, "cores": 1, "kind": "oracle",
-            "sample": f"serial C++ oracle on {wl.name} ({per_step // S} particles): one sort + {S} "
-                      f"PIC steps, {times[0]:.1f} s on 1 host core"}
+    cores = host_cores()
+    t1, per_step = run_oracle_steps(wl, 1, S, ORDERS[args.order], 1)
+    tn, _ = run_oracle_steps(wl, 1, S, ORDERS[args.order], cores)
+    one = per_step / t1[0]
+    alln = per_step / tn[0]
+    return {"value": alln, "unit": UNIT, "cores": cores, "kind": "oracle", "cpu_model": cpu_model(),
+            "single_core": {"value": one, "unit": UNIT, "cores": 1},
+            "per_core_all": alln / cores,
+            "sample": f"C++ oracle on {wl.name} ({per_step // S} particles): one sort (serial) + {S} "
+                      f"PIC steps; {tn[0]:.1f} s with the push on {cores} cores (OpenMP particle blocks, "
+                      f"private accumulators), {t1[0]:.1f} s serial on 1 core"}
 
 
 # ---------------------------------------------------------------- ours --
@@ -240,12 +295,18 @@ def our_arm(args, rank, world):
     # N > 1: weak scaling on configs[3] (C2 per GPU), or strong scaling of
     # the LPI slab (configs[4], --config 4: the 512x256x256 box split over
     # the process grid)
-    strong = world > 1 and args.config == 4
+    strong = world > 1 and args.config in STRONG_CONFIGS
     wl = inputs.config(effective_config(args, world))
     S = args.sort_every or wl.sort_every
     order = ORDERS[args.order]
+    box = wl.grid
     if strong:
         g = inputs.strong_decompose(wl.grid, world, rank)
+    elif world == 1 and args.block_of > 1:
+        # rank 0's block of a block_of-way split, its faces wrapped locally:
+        # one strong-scaling point's per-GPU compute without the exchange
+        g = inputs.strong_decompose(wl.grid, args.block_of, 0)
+        g = replace_grid(g, nbr_rank=(0,) * 6, rank=0)
     else:
         g = inputs.decompose(wl.grid, world, rank) if world > 1 else wl.grid
     from dataclasses import replace
@@ -279,6 +340,8 @@ def our_arm(args, rank, world):
                  single_round=args.migration in ("auto", "single") and (world > 1 or args.loopback))
     hp.ctx.set_option(vpic.VPIC_OPT_ADVANCE_KERNEL, {"auto": 0, "direct": 1, "tma": 2}[args.kernel])
     n_local = hp.n_particles
+    comm = {"nranks": world, "vpic_ctx_nranks": int(hp.ctx.info()["nranks"]),
+            "backend": dist.get_backend() if world > 1 else None}
 
     def barrier():
         if world > 1:
@@ -331,15 +394,18 @@ def our_arm(args, rank, world):
         sort_ms.setdefault(name, []).append(a.elapsed_time(b))
     sort_ms = {k: round(sum(v) / len(v), 3) for k, v in sort_ms.items()}
     adv_np = sum(n for _, n in adv) / len(adv)
-    t = torch.tensor([ms, float(pushes_local), float(n_local)], dtype=torch.float64, device=dev)
+    t = torch.tensor([ms, float(pushes_local), float(n_local), float(hp.n_particles)],
+                     dtype=torch.float64, device=dev)
     if world > 1:
         tmax = t.clone()
         dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
         tsum = t.clone()
         dist.all_reduce(tsum, op=dist.ReduceOp.SUM)
-        ms_max, pushes, ntot = float(tmax[0]), float(tsum[1]), float(tsum[2])
+        ms_max, pushes, ntot, nend = float(tmax[0]), float(tsum[1]), float(tsum[2]), float(tsum[3])
     else:
-        ms_max, pushes, ntot = ms, float(pushes_local), float(n_local)
+        ms_max, pushes, ntot, nend = ms, float(pushes_local), float(n_local), float(hp.n_particles)
+    # global particle count: conserved by every exchange (no absorbing walls here)
+    conservation = {"particles_start": int(ntot), "particles_end": int(nend), "ok": int(ntot) == int(nend)}
     value = pushes / (ms_max / 1e3)
 
     # ---- e2e: host (pinned) -> device inputs and device -> host results inside the timed region.
@@ -408,7 +474,10 @@ def our_arm(args, rank, world):
                    "deposit": args.deposit if args.deposit != "auto" else
                    "auto (warp; smem per species while its thermal spread since the sort is 0.4-1.3 cells)",
                    "kernel": args.kernel,
-                   "parallelism": "loopback1" if args.loopback and world == 1 else f"domain{world}",
+                   "parallelism": ("loopback1" if args.loopback and world == 1 else
+                                   f"block 0 of {args.block_of} (1 GPU, no exchange)" if world == 1 and args.block_of > 1
+                                   else f"domain{world}"),
+                   "box_cells": [box.nx, box.ny, box.nz],
                    "field_solve": bool(args.field_solve),
                    "exchange": ("nccl" if args.exchange == "nccl" else "device")
                                if (world > 1 or args.loopback) else "none",
@@ -427,6 +496,8 @@ def our_arm(args, rank, world):
                      "avg_launch_ms_by_step_since_sort": by_step,
                      "launch_ms_by_species_step": by_species},
         "sort_ms_by_species": sort_ms,
+        "comm": comm,
+        "conservation": conservation,
         "clocks": clocks,
         "gpu_launches": launches,
         "e2e": e2e,
@@ -437,6 +508,30 @@ def our_arm(args, rank, world):
     print(json.dumps(out), flush=True)
 
 
+def replace_grid(g, **kw):
+    from dataclasses import replace
+    return replace(g, **kw)
+
+
+def spawn_ranks(n: int) -> int:
+    """`bench.py --gpus N` without a torchrun environment: launch N ranks
+    (one per GPU, NCCL) through torch.distributed.run on 127.0.0.1 and
+    return their exit code; rank 0 prints the JSON line."""
+    import socket
+    import torch
+    have = torch.cuda.device_count()
+    if have < n:
+        print(f"bench.py: --gpus {n} but {have} GPU(s) visible", file=sys.stderr, flush=True)
+        return 2
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    print(f"bench.py: launching {n} ranks: {' '.join(cmd)}", file=sys.stderr, flush=True)
+    return subprocess.call(cmd)
+
+
 def main():
     args = parse()
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -444,11 +539,16 @@ def main():
     if args.impl == "reference":
         reference_arm(args, rank, world)
         return
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(spawn_ranks(args.gpus))
     if world > 1:
         import torch
         import torch.distributed as dist
         torch.cuda.set_device(int(os.environ.get("LOCAL_RANK", "0")))
         dist.init_process_group("nccl")
+        if rank == 0:
+            print(f"bench.py: NCCL process group initialised, nranks={dist.get_world_size()}",
+                  file=sys.stderr, flush=True)
     try:
         our_arm(args, rank, world)
     finally:

@@ -38,10 +38,11 @@ class OrcGrid(ctypes.Structure):
 
 
 def build(force: bool = False) -> str:
-    """Compile liboracle.so (g++ -O2 -ffp-contract=off: no FMA contraction)."""
+    """Compile liboracle.so (g++ -O2 -ffp-contract=off: no FMA contraction;
+    -fopenmp for the all-core baseline orc_advance_p_omp only)."""
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < max(
             os.path.getmtime(_SRC), os.path.getmtime(os.path.join(_HERE, "vpic_oracle.h"))):
-        cmd = ["g++", "-O2", "-std=c++17", "-ffp-contract=off", "-fno-fast-math",
+        cmd = ["g++", "-O2", "-std=c++17", "-ffp-contract=off", "-fno-fast-math", "-fopenmp",
                "-fPIC", "-shared", _SRC, "-o", _LIB + ".tmp"]
         subprocess.check_call(cmd)
         os.replace(_LIB + ".tmp", _LIB)
@@ -66,6 +67,9 @@ def lib() -> ctypes.CDLL:
         _lib.orc_load_interpolator.restype = None
         _lib.orc_advance_p.argtypes = [G, ctypes.c_float, ctypes.c_float, P, I64, P, P, P, P, P, I64]
         _lib.orc_advance_p.restype = I64
+        _lib.orc_advance_p_omp.argtypes = [G, ctypes.c_float, ctypes.c_float, P, I64, P, P, P, I64,
+                                           ctypes.c_int]
+        _lib.orc_advance_p_omp.restype = I64
         _lib.orc_move_deposit.argtypes = [G, ctypes.c_float, P, I64, P, P, P, P, I64]
         _lib.orc_move_deposit.restype = I64
         _lib.orc_move_p.argtypes = [G, P, P, P, P, P, ctypes.c_float]
@@ -156,6 +160,21 @@ def advance_p(spec, q, m, p, interp, acc, acc_abs=None, max_movers=None, acc_con
     g = make_grid(spec)
     nm = lib().orc_advance_p(ctypes.byref(g), q, m, _ptr(p), p.size, _ptr(interp), _ptr(acc),
                              _ptr(acc_abs), _ptr(acc_cond), _ptr(movers), max_movers)
+    if nm < 0:
+        raise OverflowError("mover list overflow")
+    return movers[:nm].copy()
+
+
+def advance_p_omp(spec, q, m, p, interp, acc, threads, max_movers=None):
+    """advance_p over `threads` particle blocks (OpenMP, private accumulators)."""
+    assert p.dtype == PARTICLE_DTYPE and p.flags.c_contiguous
+    assert acc.dtype == np.float32 and acc.flags.c_contiguous
+    if max_movers is None:
+        max_movers = p.size
+    movers = np.zeros(max(max_movers, 1), MOVER_DTYPE)
+    g = make_grid(spec)
+    nm = lib().orc_advance_p_omp(ctypes.byref(g), q, m, _ptr(p), p.size, _ptr(interp), _ptr(acc),
+                                 _ptr(movers), max_movers, int(threads))
     if nm < 0:
         raise OverflowError("mover list overflow")
     return movers[:nm].copy()

@@ -67,6 +67,14 @@ int64_t orc_advance_p(const orc_grid *g, float q, float m, orc_particle *p, int6
                       const float *interp, float *acc, double *acc_abs, double *acc_cond,
                       orc_mover *movers, int64_t max_movers);
 
+/* orc_advance_p over nthreads contiguous particle blocks (OpenMP), each with
+ * a private accumulator summed into acc afterwards (the all-core CPU
+ * baseline).  Same particles as orc_advance_p; acc equal up to summation
+ * order; movers in block order. */
+int64_t orc_advance_p_omp(const orc_grid *g, float q, float m, orc_particle *p, int64_t np,
+                          const float *interp, float *acc, orc_mover *movers, int64_t max_movers,
+                          int nthreads);
+
 /* The move-and-deposit half of orc_advance_p alone: p[].u must already be
  * the pushed momentum (replay of another implementation's momenta). */
 int64_t orc_move_deposit(const orc_grid *g, float qsp, orc_particle *p, int64_t np, float *acc,

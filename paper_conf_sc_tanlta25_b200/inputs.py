@@ -118,6 +118,15 @@ def config(idx: int) -> Workload:
         return Workload("lpi_slab512x256x256_ppc64", GridSpec(512, 256, 256),
                         [Species("electron", -1.0, 1.0, 0.2, (0.3, 0.0, 0.0)),
                          Species("ion", 1.0, 1836.0, 0.002)], 64, 100, 20, kind="lpi")
+    if idx == 5:
+        # the paper's strong-scaling regime (Fig. 9/10,
+        # sorting disabled, per-GPU grids shrinking into
+        # the cache).  256x128x128 cells: interpolator + accumulator 628 MB >>
+        # the 126 MB L2 on one GPU, 81 MB per GPU on 8 (2x2x2 blocks of
+        # 128x64x64).  Random (shuffled) order, no sort.
+        return Workload("f3_l2strong_uniform256x128x128_ppc32_nosort", GridSpec(256, 128, 128),
+                        [e(), Species("ion", 1.0, 25.0, 0.02)], 32, 100, 20,
+                        notes="order none + shuffled")
     raise IndexError(idx)
 
 
@@ -288,15 +297,19 @@ def decompose(block: GridSpec, nranks: int, rank: int) -> GridSpec:
         cc = [cc[a] % P[a] for a in range(3)]
         return cc[0] + P[0] * (cc[1] + P[1] * cc[2])
 
-    nbr = []
+    nbr, pbc = [], []
     for f in range(6):
         a = f % 3
         d = -1 if f < 3 else 1
         cc = list(c)
         cc[a] += d
         nbr.append(rank_of(cc))
+        # the box's own wall (reflect / absorb) only on its outer faces; faces
+        # between blocks are periodic (remote)
+        outer = cc[a] < 0 or cc[a] >= P[a]
+        pbc.append(block.pbc[f] if outer else BC_PERIODIC)
     n = (block.nx, block.ny, block.nz)
-    return replace(block, nbr_rank=tuple(nbr), rank=rank,
+    return replace(block, nbr_rank=tuple(nbr), pbc=tuple(pbc), rank=rank,
                    gx0=c[0] * n[0], gy0=c[1] * n[1], gz0=c[2] * n[2])
 
 
@@ -311,3 +324,47 @@ def strong_decompose(box: GridSpec, nranks: int, rank: int) -> GridSpec:
     block = replace(box, nx=box.nx // P[0], ny=box.ny // P[1], nz=box.nz // P[2],
                     gnx=box.gnx or box.nx)
     return decompose(block, nranks, rank)
+
+
+# ------------------------------------------------ block <-> global views --
+def _block_coords(gg: GridSpec, gb: GridSpec, X, Y, Z):
+    """Global interior cell coordinates -> block-local ones (may fall outside)."""
+    return X - gb.gx0, Y - gb.gy0, Z - gb.gz0
+
+
+def to_block(gg: GridSpec, gb: GridSpec, p: np.ndarray) -> np.ndarray:
+    """The particles of the global box gg (voxels indexed on gg) that lie in
+    block gb (a decompose()/strong_decompose() block of gg), re-indexed on gb."""
+    X, Y, Z = gg.coords(p["i"])
+    x, y, z = _block_coords(gg, gb, X, Y, Z)
+    m = (x >= 1) & (x <= gb.nx) & (y >= 1) & (y <= gb.ny) & (z >= 1) & (z <= gb.nz)
+    out = p[m].copy()
+    out["i"] = gb.voxel(x[m], y[m], z[m]).astype(np.int32)
+    return out
+
+
+def to_global(gg: GridSpec, gb: GridSpec, p: np.ndarray) -> np.ndarray:
+    """Block-indexed particles back on the global box's voxel indices."""
+    x, y, z = gb.coords(p["i"])
+    out = p.copy()
+    out["i"] = gg.voxel(x + gb.gx0, y + gb.gy0, z + gb.gz0).astype(np.int32)
+    return out
+
+
+def block_fields(gg: GridSpec, gb: GridSpec, f: np.ndarray) -> np.ndarray:
+    """fields[nv_block][8] of block gb cut from the global fields (interior and
+    ghost voxels; ghost coordinates wrap periodically on the global box)."""
+    v = np.arange(gb.nv)
+    x, y, z = gb.coords(v)
+    n = (gg.nx, gg.ny, gg.nz)
+    X = (x + gb.gx0 - 1) % n[0] + 1
+    Y = (y + gb.gy0 - 1) % n[1] + 1
+    Z = (z + gb.gz0 - 1) % n[2] + 1
+    return f[gg.voxel(X, Y, Z)].copy()
+
+
+def block_interior_to_global(gg: GridSpec, gb: GridSpec) -> Tuple[np.ndarray, np.ndarray]:
+    """(block voxel, global voxel) index pairs of the block's interior."""
+    vb = gb.interior_voxels().astype(np.int64)
+    x, y, z = gb.coords(vb)
+    return vb, gg.voxel(x + gb.gx0, y + gb.gy0, z + gb.gz0).astype(np.int64)

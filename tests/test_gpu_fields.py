@@ -88,16 +88,51 @@ def _multiset(a):
     return np.sort(np.ascontiguousarray(a).view(np.dtype((np.void, 32))).ravel())
 
 
+def oracle_steps(orc, g, wl, parts, fields, steps, field_solve=False, eps0=1.0):
+    """The single-domain oracle run of `steps` PIC steps (locally periodic
+    faces, walls as in g; absorbed particles removed by back-fill): returns
+    the particles per species, the last step's jf and its per-edge sum of
+    |contributions| (the T1 weights of jf)."""
+    po = [p.copy() for p in parts]
+    fo = fields.copy()
+    for _ in range(steps):
+        interp = orc.load_interpolator(g, fo)
+        acc = np.zeros((g.nv, 12), np.float32)
+        aabs = np.zeros((g.nv, 12), np.float64)
+        for k, sp in enumerate(wl.species):
+            mv = orc.advance_p(g, sp.q, sp.m, po[k], interp, acc, aabs)
+            if mv.size:
+                po[k] = orc.remove_absorbed(g, po[k], mv)
+        jf = orc.unload_accumulator(g, acc)
+        if field_solve:
+            orc.advance_b(g, fo, 0.5)
+            orc.advance_e(g, fo, jf, eps0)
+            orc.advance_b(g, fo, 0.5)
+    jf_abs = orc.unload_accumulator(g, aabs.astype(np.float32)).astype(np.float64)
+    return po, jf, jf_abs, fo
+
+
+def assert_jf_t1(g, jf_gpu, jf_orc, jf_abs):
+    """T1 on the unloaded currents: per edge |jf_gpu - jf_orc| <= 1e-5 x the
+    unloaded sum of |contributions| (periodic fold included)."""
+    vox = g.interior_voxels()
+    err = np.abs(jf_gpu[vox, :3].astype(np.float64) - jf_orc[vox, :3])
+    tol = 1e-5 * jf_abs[vox, :3] + 1e-30
+    assert (err <= tol).all(), f"{(err > tol).sum()} jf entries beyond T1, worst {err.max()}"
+
+
 @pytest.mark.parametrize("walls", [False, True], ids=["periodic", "reflect_z"])
 @pytest.mark.parametrize("migration", ["rounds", "single"])
 @pytest.mark.parametrize("device_exchange", [False, True], ids=["nccl", "device"])
 @pytest.mark.parametrize("field_solve,steps", [(False, 3), (True, 1)])
-def test_loopback_exchange_matches_periodic(V, field_solve, steps, device_exchange, migration, walls):
+def test_loopback_exchange_matches_oracle(V, orc, field_solve, steps, device_exchange, migration, walls):
     """VPIC_OPT_LOOPBACK_EXCHANGE sends every periodic crossing, E/cB halo and
     jf shared plane through the NCCL exchange (one-rank communicator, self
-    peer): the multi-GPU code path on one GPU.  It must reproduce the local
-    periodic wrap: particles bit-exact as multisets (migration reorders
-    them), jf and fields within the atomic-reordering tolerance.  "device":
+    peer): the multi-GPU code path on one GPU.  Compared with the ORACLE's
+    single-domain run (IEEE math): particles bit-exact as multisets
+    (migration reorders them), jf per edge within T1 of the oracle's, fields
+    bit-exact when static (halos move bytes only) and within the jf
+    tolerance propagated through the field solve otherwise.  "device":
     the device-initiated exchange (f4) -- the push stores movers into the
     (self) neighbour's symmetric-memory inbox, rounds synchronised on the
     device.  "single": VPIC_OPT_SINGLE_ROUND_MIGRATION -- moves finished in
@@ -121,25 +156,29 @@ def test_loopback_exchange_matches_periodic(V, field_solve, steps, device_exchan
         torch.cuda.synchronize()
         runs.append(hp)
     a, b = runs
+    po, jo, jabs, fo = oracle_steps(orc, g, wl, parts, fields, steps, field_solve)
     for k in range(2):
         pa, pb = a.particles_host(k), b.particles_host(k)
         assert pa.size == pb.size == parts[k].size
-        assert np.array_equal(_multiset(pa), _multiset(pb))
+        assert np.array_equal(_multiset(pb), _multiset(po[k]))    # loopback exchange vs oracle
+        assert np.array_equal(_multiset(pa), _multiset(po[k]))    # local wrap vs oracle
         # migration really ran: departed particles were back-filled, arrivals appended
         assert not np.array_equal(pa.view(np.uint32), pb.view(np.uint32))
+    assert_jf_t1(g, b.jf.cpu().numpy(), jo, jabs)
+    assert_jf_t1(g, a.jf.cpu().numpy(), jo, jabs)
     vox = g.interior_voxels()
-    ja, jb = a.jf.cpu().numpy()[vox], b.jf.cpu().numpy()[vox]
-    assert np.abs(ja - jb).max() <= 1e-5 * np.abs(ja).max() * 8
-    fa, fb = a.fields.cpu().numpy()[vox], b.fields.cpu().numpy()[vox]
-    assert np.abs(fa - fb).max() <= 1e-5 * max(1.0, np.abs(fa).max())
+    fb = b.fields.cpu().numpy()[vox]
     if not field_solve:
-        assert np.array_equal(fa, fb)       # static fields: halos move bytes only
+        assert np.array_equal(fb, fo[vox])       # static fields: halos move bytes only
+    else:   # E carries -dt/eps0 jf: T1 of jf, carried once through curl E into cB
+        tol = 1e-5 * g.dt * jabs.max() * 4 + 1e-6 * np.abs(fo).max()
+        assert np.abs(fb.astype(np.float64) - fo[vox]).max() <= tol
 
 
 @pytest.mark.parametrize("walls", [False, True], ids=["periodic", "absorb_z"])
 @pytest.mark.parametrize("migration", ["rounds", "single"])
 @pytest.mark.parametrize("device_exchange", [False, True], ids=["nccl", "device"])
-def test_loopback_direct_kernel_matches_periodic(V, device_exchange, migration, walls):
+def test_loopback_direct_kernel_matches_oracle(V, orc, device_exchange, migration, walls):
     """As above with the direct-load advance kernel (VPIC_OPT_ADVANCE_KERNEL =
     1): its crossers leave through the same move_p / leave() code.  absorb_z:
     absorbing z walls -- particles that enter the ghost layer through x/y and
@@ -160,14 +199,15 @@ def test_loopback_direct_kernel_matches_periodic(V, device_exchange, migration, 
         torch.cuda.synchronize()
         runs.append(hp)
     a, b = runs
+    po, jo, jabs, _ = oracle_steps(orc, g, wl, parts, fields, 2)
     pa, pb = a.particles_host(0), b.particles_host(0)
     if walls:
         assert pa.size < parts[0].size          # some were absorbed
-    assert np.array_equal(_multiset(pa), _multiset(pb))
+    assert np.array_equal(_multiset(pb), _multiset(po[0]))
+    assert np.array_equal(_multiset(pa), _multiset(po[0]))
     assert not np.array_equal(pa.view(np.uint32), pb.view(np.uint32))
-    vox = g.interior_voxels()
-    ja, jb = a.jf.cpu().numpy()[vox], b.jf.cpu().numpy()[vox]
-    assert np.abs(ja - jb).max() <= 1e-5 * np.abs(ja).max() * 8
+    assert_jf_t1(g, b.jf.cpu().numpy(), jo, jabs)
+    assert_jf_t1(g, a.jf.cpu().numpy(), jo, jabs)
 
 
 @pytest.mark.parametrize("migration", ["rounds", "single"])

@@ -425,3 +425,28 @@ def test_single_round_protocol_eight_ranks():
         assert np.all(acc[ghost] == 0)
         got = acc[1:-1, 1:-1, 1:-1]
         assert np.array_equal(got, want[z0:z0 + SB[2], y0:y0 + SB[1], x0:x0 + SB[0]]), r
+
+
+@pytest.mark.parametrize("nranks", [2, 4, 8])
+def test_block_split_roundtrip(nranks):
+    """The block views the multi-GPU parity test uses (tests/multirank_worker.py):
+    splitting a global box's particles / fields over the process grid and
+    mapping them back recovers every particle exactly once and every
+    interior field value."""
+    from paper_conf_sc_tanlta25_b200 import inputs
+    gg = inputs.GridSpec(16, 8, 8, dt=0.5)
+    wl = inputs.Workload("split", gg, [inputs.Species("electron", -1.0, 1.0, 0.6)], 5, 1, 0)
+    p = inputs.make_species_particles(wl)[0]
+    f = inputs.make_fields(gg, 0.05)
+    back, cover = [], np.zeros(gg.nv, int)
+    for r in range(nranks):
+        gb = inputs.strong_decompose(gg, nranks, r)
+        pb = inputs.to_block(gg, gb, p)
+        back.append(inputs.to_global(gg, gb, pb))
+        fb = inputs.block_fields(gg, gb, f)
+        vb, vg = inputs.block_interior_to_global(gg, gb)
+        assert np.array_equal(fb[vb], f[vg])
+        cover[vg] += 1
+    key = lambda a: np.sort(np.ascontiguousarray(a).view(np.dtype((np.void, 32))))
+    assert np.array_equal(key(np.concatenate(back)), key(p))
+    assert np.array_equal(cover[gg.interior_voxels()], np.ones(gg.ncells, int))

@@ -399,3 +399,24 @@ def test_move_deposit_replays_advance(orc):
     assert np.array_equal(pr.view(np.uint32), p1.view(np.uint32))
     assert np.array_equal(acc_r.view(np.uint32), acc.view(np.uint32))
     assert np.array_equal(mv_r.view(np.uint32), mv.view(np.uint32)) and mv.size > 0
+
+
+@pytest.mark.parametrize("threads", [1, 3, 8])
+def test_advance_p_omp_matches_serial(orc, threads):
+    """The all-core baseline (orc_advance_p_omp: particle blocks, private
+    accumulators) computes the serial oracle's step: particles bit-exact,
+    accumulator equal up to summation order, same movers."""
+    g = inputs.GridSpec(6, 5, 4, dt=0.5, pbc=(0, 0, 2, 0, 0, 2))
+    p = inputs.random_particles(g, 5001, 23, u_scale=1.0)
+    interp = orc.load_interpolator(g, (np.random.default_rng(4).random((g.nv, 8), np.float32) - 0.5) * 0.2)
+    a1 = np.zeros((g.nv, 12), np.float32)
+    aa = np.zeros((g.nv, 12), np.float64)
+    p1 = p.copy()
+    m1 = orc.advance_p(g, -1.0, 1.0, p1, interp, a1, aa)
+    a2 = np.zeros_like(a1)
+    p2 = p.copy()
+    m2 = orc.advance_p_omp(g, -1.0, 1.0, p2, interp, a2, threads)
+    assert np.array_equal(p1.view(np.uint32), p2.view(np.uint32))
+    assert np.all(np.abs(a1.astype(np.float64) - a2) <= 1e-5 * aa + 1e-30)
+    assert np.array_equal(np.sort(m1.view(np.uint32).reshape(-1, 4), axis=0),
+                          np.sort(m2.view(np.uint32).reshape(-1, 4), axis=0)) and m1.size > 0

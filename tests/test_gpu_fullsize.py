@@ -99,7 +99,9 @@ def test_fullsize_sort_properties(state, order):
     perm = torch.empty(n, dtype=torch.int64, device="cuda")
     counts = torch.empty(g.nv, dtype=torch.int32, device="cuda")
     T = hp.ctx.info()["tile_sz"]
-    vpic.vpic_sort_particles(hp.ctx, p_in, out, n, order, 0, hp.ws, counts, None, perm)
+    ws = torch.empty(vpic.vpic_sort_workspace_bytes(hp.ctx, n, order), dtype=torch.uint8, device="cuda")
+    vpic.vpic_sort_particles(hp.ctx, p_in, out, n, order, 0, ws, counts, None, perm)
+    del ws
     torch.cuda.synchronize()
     # a permutation, payload moved with it, counts consistent
     assert torch.equal(torch.sort(perm).values, torch.arange(n, device="cuda"))

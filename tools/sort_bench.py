@@ -23,7 +23,7 @@ a = ap.parse_args()
 order = {"standard": 0, "strided": 1, "tiled_strided": 2}[a.order]
 wl = inputs.config(a.config)
 parts = inputs.make_species_particles(wl)
-hp = HotPath(wl, parts, inputs.make_fields(wl.grid, wl.field_amp))
+hp = HotPath(wl, parts, inputs.make_fields(wl.grid, wl.field_amp), order=order)
 for _ in range(a.steps):
     hp.step()
 torch.cuda.synchronize()

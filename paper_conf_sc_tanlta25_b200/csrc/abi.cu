@@ -2,6 +2,7 @@
 // context, and dispatch to the kernels.  No C++ exception crosses the ABI
 // and nothing aborts; every entry point returns a vpic_status.
 #include <nccl.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include <atomic>
 #include <cstring>
@@ -30,6 +31,14 @@ bool grid_ok(const vpic_grid_t *g) {
     if (g->pbc[f] < 0 || g->pbc[f] > 2) return false;
   return true;
 }
+
+// One NVTX range per C-ABI call (SURVEY.md §5 tracing): visible in nsys /
+// ncu --nvtx timelines; a no-op without an attached tool.
+struct NvtxRange {
+  explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
+#define VPIC_NVTX() NvtxRange nvtx_range_(__func__)
 
 struct DeviceGuard {
   int prev = -1;
@@ -86,6 +95,7 @@ int vpic_get_unique_id(uint8_t uid[128]) {
 
 int vpic_ctx_create(vpic_ctx **out, const vpic_grid_t *g, int rank, int nranks,
                     const uint8_t *uid, int device) {
+  VPIC_NVTX();
   if (!out || !grid_ok(g) || nranks < 1 || rank < 0 || rank >= nranks) return VPIC_ERR_INVALID;
   *out = nullptr;
   for (int f = 0; f < 6; ++f) {
@@ -151,6 +161,7 @@ int vpic_ctx_create(vpic_ctx **out, const vpic_grid_t *g, int rank, int nranks,
 }
 
 int vpic_ctx_destroy(vpic_ctx *c) {
+  VPIC_NVTX();
   if (!c) return VPIC_ERR_INVALID;
   DeviceGuard dg(c->device);
   exchange_destroy(c);
@@ -161,6 +172,7 @@ int vpic_ctx_destroy(vpic_ctx *c) {
 }
 
 int vpic_ctx_set_option(vpic_ctx *c, int option, int64_t value) {
+  VPIC_NVTX();
   if (!c) return VPIC_ERR_INVALID;
   switch (option) {
     case VPIC_OPT_MATH:
@@ -232,6 +244,7 @@ size_t vpic_sort_workspace_bytes(const vpic_ctx *c, int64_t np, int order) {
 int vpic_sort_particles(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_t *p_out,
                         int64_t np, int order, int64_t tile_sz, void *ws, size_t ws_bytes,
                         int32_t *voxel_counts, int64_t *new_keys, int64_t *perm, void *stream) {
+  VPIC_NVTX();
   if (!c || np < 0 || np >= ((int64_t)1 << 32) || order < 0 || order > 3 || tile_sz < 0)
     return VPIC_ERR_INVALID;
   if (np > 0 && (!p_in || !p_out || !aligned16(p_in) || !aligned16(p_out))) return VPIC_ERR_INVALID;
@@ -246,6 +259,7 @@ int vpic_sort_particles(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_
 }
 
 int vpic_load_interpolator(vpic_ctx *c, float *fields, float *interp, void *stream) {
+  VPIC_NVTX();
   if (!c || !fields || !interp || !aligned16(fields) || !aligned32(interp)) return VPIC_ERR_INVALID;
   DeviceGuard dg(c->device);
   cudaError_t e = launch_fill_ghosts(c, fields, S(stream));
@@ -258,6 +272,7 @@ int vpic_load_interpolator(vpic_ctx *c, float *fields, float *interp, void *stre
 }
 
 int vpic_clear_accumulator(vpic_ctx *c, float *acc, void *stream) {
+  VPIC_NVTX();
   if (!c || !acc) return VPIC_ERR_INVALID;
   DeviceGuard dg(c->device);
   return cuda_status(cudaMemsetAsync(acc, 0, (size_t)c->gk.nv * 48, S(stream)));
@@ -266,6 +281,7 @@ int vpic_clear_accumulator(vpic_ctx *c, float *acc, void *stream) {
 int vpic_advance_p(vpic_ctx *c, float q, float m, vpic_particle_t *p, int64_t np,
                    const float *interp, float *acc, vpic_mover_t *movers, int64_t max_movers,
                    int64_t *n_movers, int32_t *flags, void *stream) {
+  VPIC_NVTX();
   if (!c || np < 0 || np >= ((int64_t)1 << 31) || !(m > 0) || max_movers < 0) return VPIC_ERR_INVALID;
   if (np == 0) return VPIC_OK;
   if (!p || !interp || !acc || !n_movers || !aligned16(p) || !aligned32(interp) || !aligned16(acc))
@@ -280,6 +296,7 @@ int vpic_advance_p(vpic_ctx *c, float q, float m, vpic_particle_t *p, int64_t np
 int vpic_advance_p_dev(vpic_ctx *c, float q, float m, vpic_particle_t *p, const int64_t *np_dev,
                        int64_t max_np, const float *interp, float *acc, vpic_mover_t *movers,
                        int64_t max_movers, int64_t *n_movers, int32_t *flags, void *stream) {
+  VPIC_NVTX();
   if (!c || !np_dev || max_np < 0 || max_np >= ((int64_t)1 << 31) || !(m > 0) || max_movers < 0)
     return VPIC_ERR_INVALID;
   if ((reinterpret_cast<uintptr_t>(np_dev) & 7u) != 0) return VPIC_ERR_INVALID;
@@ -294,6 +311,7 @@ int vpic_advance_p_dev(vpic_ctx *c, float q, float m, vpic_particle_t *p, const 
 }
 
 int vpic_unload_accumulator(vpic_ctx *c, const float *acc, float *jf, void *stream) {
+  VPIC_NVTX();
   if (!c || !acc || !jf || !aligned16(acc) || !aligned16(jf)) return VPIC_ERR_INVALID;
   DeviceGuard dg(c->device);
   if (cudaMemsetAsync(jf, 0, (size_t)c->gk.nv * 16, S(stream)) != cudaSuccess) return VPIC_ERR_CUDA;
@@ -304,6 +322,7 @@ int vpic_unload_accumulator(vpic_ctx *c, const float *acc, float *jf, void *stre
 }
 
 int vpic_advance_b(vpic_ctx *c, float *fields, float frac, void *stream) {
+  VPIC_NVTX();
   if (!c || !fields || !aligned16(fields) || !(frac >= 0)) return VPIC_ERR_INVALID;
   DeviceGuard dg(c->device);
   if (launch_fill_ghosts(c, fields, S(stream)) != cudaSuccess) return VPIC_ERR_CUDA;
@@ -315,6 +334,7 @@ int vpic_advance_b(vpic_ctx *c, float *fields, float frac, void *stream) {
 }
 
 int vpic_advance_e(vpic_ctx *c, float *fields, const float *jf, float eps0, void *stream) {
+  VPIC_NVTX();
   if (!c || !fields || !jf || !aligned16(fields) || !aligned16(jf) || !(eps0 > 0))
     return VPIC_ERR_INVALID;
   DeviceGuard dg(c->device);
@@ -328,6 +348,7 @@ int vpic_advance_e(vpic_ctx *c, float *fields, const float *jf, float eps0, void
 
 int vpic_accumulate_rho(vpic_ctx *c, float q, const vpic_particle_t *p, int64_t np, float *rho,
                         void *stream) {
+  VPIC_NVTX();
   if (!c || np < 0 || !rho || (np > 0 && (!p || !aligned16(p)))) return VPIC_ERR_INVALID;
   DeviceGuard dg(c->device);
   return cuda_status(launch_accumulate_rho(c, q, p, np, rho, S(stream)));
@@ -335,6 +356,7 @@ int vpic_accumulate_rho(vpic_ctx *c, float q, const vpic_particle_t *p, int64_t 
 
 int vpic_continuity_residual(vpic_ctx *c, const float *rho0, const float *rho1, const float *jf,
                              float *out, float *res, void *stream) {
+  VPIC_NVTX();
   if (!c || !rho0 || !rho1 || !jf || !out || !aligned16(jf)) return VPIC_ERR_INVALID;
   DeviceGuard dg(c->device);
   return cuda_status(launch_continuity(c, rho0, rho1, jf, out, res, S(stream)));
@@ -343,6 +365,7 @@ int vpic_continuity_residual(vpic_ctx *c, const float *rho0, const float *rho1, 
 int vpic_gather_scatter(vpic_ctx *c, const int32_t *keys, const double *x, int64_t n,
                         const double *table, double *out, double *acc, int64_t nkeys,
                         int64_t stencil_nx, int aggregate, void *stream) {
+  VPIC_NVTX();
   if (!c || n < 0 || nkeys <= 0 || nkeys >= ((int64_t)1 << 31) || stencil_nx < 0) return VPIC_ERR_INVALID;
   if (n > 0 && (!keys || !x || !table || !out || !acc)) return VPIC_ERR_INVALID;
   DeviceGuard dg(c->device);
@@ -353,6 +376,7 @@ int vpic_gather_scatter(vpic_ctx *c, const int32_t *keys, const double *x, int64
 int vpic_migrate_particles(vpic_ctx *c, float q, float m, vpic_particle_t *p, int64_t *np,
                            int64_t max_np, vpic_mover_t *movers, int64_t max_movers,
                            const int64_t *n_movers, float *acc, void *stream) {
+  VPIC_NVTX();
   if (!c || !np || *np < 0 || max_np < *np || !n_movers || !acc || max_movers < 0)
     return VPIC_ERR_INVALID;
   if (max_np >= ((int64_t)1 << 31)) return VPIC_ERR_INVALID;
@@ -366,6 +390,7 @@ int vpic_migrate_particles_dev(vpic_ctx *c, float q, float m, vpic_particle_t *p
                                int64_t max_np, const vpic_mover_t *movers, int64_t max_movers,
                                const int64_t *n_movers, float *acc, int32_t *flags_dev,
                                void *stream) {
+  VPIC_NVTX();
   (void)q; (void)m;
   if (!c || !np_dev || max_np < 0 || max_np >= ((int64_t)1 << 31) || !n_movers || !acc || !p ||
       !aligned16(p) || !flags_dev || max_movers < 0)

@@ -27,10 +27,12 @@ def _ngpu():
 
 
 @pytest.mark.timeout(900)
-@pytest.mark.parametrize("nranks", [2, 4, 8])
-def test_multirank_exchange_matches_oracle(orc, tmp_path, nranks):
-    if _ngpu() < nranks:
-        pytest.skip(f"needs {nranks} GPUs, {_ngpu()} visible")
+def test_multirank_exchange_matches_oracle(orc, tmp_path):
+    """On as many GPUs as the box has (8, 4 or 2: process grids 2x2x2,
+    2x2x1, 2x1x1)."""
+    nranks = max([n for n in (2, 4, 8) if n <= _ngpu()], default=0)
+    if nranks == 0:
+        pytest.skip(f"needs >= 2 GPUs, {_ngpu()} visible")
     sys.path.insert(0, HERE)
     import multirank_worker as W
     from paper_conf_sc_tanlta25_b200 import _build

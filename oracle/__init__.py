@@ -70,6 +70,8 @@ def lib() -> ctypes.CDLL:
         _lib.orc_advance_p_omp.argtypes = [G, ctypes.c_float, ctypes.c_float, P, I64, P, P, P, I64,
                                            ctypes.c_int]
         _lib.orc_advance_p_omp.restype = I64
+        _lib.orc_continuity_residual.argtypes = [G, P, P, P, P, P]
+        _lib.orc_continuity_residual.restype = None
         _lib.orc_move_deposit.argtypes = [G, ctypes.c_float, P, I64, P, P, P, P, I64]
         _lib.orc_move_deposit.restype = I64
         _lib.orc_move_p.argtypes = [G, P, P, P, P, P, ctypes.c_float]
@@ -224,6 +226,19 @@ def accumulate_rho(spec, p, q, rho=None):
     p = np.ascontiguousarray(p, dtype=PARTICLE_DTYPE)
     lib().orc_accumulate_rho(ctypes.byref(g), _ptr(p), p.size, q, _ptr(rho))
     return rho
+
+
+def continuity_residual(spec, rho0, rho1, jf):
+    """(res, mag) per node, float64[nv] (NaN outside the node range): the
+    discrete continuity residual of float32 rho0/rho1[nv], jf[nv,4] (D1)."""
+    rho0 = np.ascontiguousarray(rho0, np.float32)
+    rho1 = np.ascontiguousarray(rho1, np.float32)
+    jf = np.ascontiguousarray(jf, np.float32)
+    res = np.full(rho0.size, np.nan)
+    mag = np.full(rho0.size, np.nan)
+    g = make_grid(spec)
+    lib().orc_continuity_residual(ctypes.byref(g), _ptr(rho0), _ptr(rho1), _ptr(jf), _ptr(res), _ptr(mag))
+    return res, mag
 
 
 def remove_absorbed(spec, p, movers):

@@ -86,6 +86,13 @@ int64_t orc_move_deposit(const orc_grid *g, float qsp, orc_particle *p, int64_t 
 int orc_move_p(const orc_grid *g, orc_particle *p, orc_mover *pm, float *acc,
                double *acc_abs, double *acc_cond, float qsp);
 
+/* Discrete continuity residual per node (reading D1), in double:
+ * res = (rho1-rho0)/(dV dt) + sum_a (jf_a(n) - jf_a(n - e_a))/d_a over nodes
+ * 1..n (locally periodic axis, n - e wraps) or 1..n+1; other entries of res
+ * untouched.  mag (nullable): sum of the terms' absolute values. */
+void orc_continuity_residual(const orc_grid *g, const float *rho0, const float *rho1,
+                             const float *jf, double *res, double *mag);
+
 /* jf[nv][4] (jfx,jfy,jfz,0) from acc[nv][12]; locally periodic planes folded. */
 void orc_unload_accumulator(const orc_grid *g, const float *acc, float *jf);
 

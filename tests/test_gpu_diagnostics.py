@@ -69,7 +69,7 @@ def test_rho_empty_and_invalid(V):
         V.vpic_accumulate_rho(ctx, 1.0, None, 4, rho)
 
 
-def advance_with_residual(V, g, p, q, fields, perturb=1.0):
+def advance_with_residual(V, g, p, q, fields, perturb=1.0, arrays=False):
     ctx = V.Context(g)
     ctx.set_option(V.VPIC_OPT_MATH, V.MATH_FAST)
     fd = torch.from_numpy(fields.copy()).cuda()
@@ -93,6 +93,9 @@ def advance_with_residual(V, g, p, q, fields, perturb=1.0):
     res = torch.full((g.nv,), 7.0, dtype=torch.float32, device="cuda")
     V.vpic_continuity_residual(ctx, rho0, rho1, jf, out, res)
     torch.cuda.synchronize()
+    if arrays:
+        return (out.cpu().numpy().astype(np.float64), res.cpu().numpy(), rho0.cpu().numpy(),
+                rho1.cpu().numpy(), jf.cpu().numpy())
     return out.cpu().numpy().astype(np.float64), res.cpu().numpy(), int(nm.item())
 
 
@@ -120,3 +123,22 @@ def test_continuity_residual_detects_wrong_current(V):
     out, _, _ = advance_with_residual(V, g, p, 0.7, inputs.make_fields(g, 0.05), perturb=1.01)
     assert out[0] > 3e-3 * out[1]
 
+
+
+@pytest.mark.parametrize("pbc", [(0,) * 6, (0, 0, 1, 0, 0, 1)], ids=["periodic", "reflect_z"])
+def test_continuity_residual_parity(V, orc, pbc):
+    """vpic_continuity_residual against the oracle's definition
+    (orc_continuity_residual, reading D1) on the same float32 rho0 / rho1 /
+    jf: per node within 4 float32 roundings of the terms' magnitude, the
+    same node range, the max reductions equal to the maxima of the arrays."""
+    g = inputs.GridSpec(8, 6, 5, dx=0.8, dy=1.0, dz=1.25, dt=0.4, pbc=pbc)
+    p = inputs.random_particles(g, 60000, 23, u_scale=0.8)
+    out, res, rho0, rho1, jf = advance_with_residual(V, g, p, 0.7, inputs.make_fields(g, 0.05), arrays=True)
+    ro, mag = orc.continuity_residual(g, rho0, rho1, jf)
+    inside = ~np.isnan(ro)
+    assert np.all(res[~inside] == 7.0)               # untouched outside the node range
+    err = np.abs(res[inside].astype(np.float64) - ro[inside])
+    assert np.all(err <= 4 * 2.0**-24 * mag[inside] + 1e-30), err.max()
+    assert out[0] == np.float32(np.abs(res[inside]).max())
+    drho = np.abs((rho1 - rho0).astype(np.float32) * np.float32(1.0 / (0.8 * 1.0 * 1.25 * 0.4)))
+    assert abs(out[1] - drho[inside].max()) <= 4 * 2.0**-24 * drho[inside].max()

@@ -330,6 +330,47 @@ int vpic_migrate_particles_dev(vpic_ctx *ctx, float q, float m, vpic_particle_t 
                                const int64_t *n_movers, float *acc, int32_t *flags_dev,
                                void *stream);
 
+/* ------------------------------------ host-buffer driver (end to end) -- */
+
+/* One species of vpic_run_host: its input in pinned HOST memory, four
+ * caller-owned DEVICE particle buffers of max_np records each (they rotate
+ * through input / sort output / next upload / previous download, so the
+ * copies of neighbouring periods overlap the compute). */
+typedef struct {
+  float q, m;                        /* charge, mass */
+  const vpic_particle_t *host_in;    /* [np] pinned host: the period's input */
+  vpic_particle_t *host_out;         /* [np] pinned host, nullable: the period's particles */
+  int64_t np, max_np;                /* records in host_in; capacity of each dev buffer */
+  vpic_particle_t *dev[4];           /* device buffers, 16-B aligned */
+} vpic_species_host_t;
+
+/* Device workspace bytes vpic_run_host needs (fields x 2, interpolator,
+ * accumulator, jf x 3, mover lists, sort workspace). */
+size_t vpic_run_host_workspace_bytes(const vpic_ctx *ctx, int nsp, const vpic_species_host_t *sp,
+                                     int order);
+
+/* n_cycles sort periods of the hot path from and to pinned host memory (the
+ * end-to-end form of the paper's push + sort loop): every
+ * period uploads each species' host_in and fields_host (nv x 8 floats),
+ * sorts every species in `order` (tile_sz as in vpic_sort_particles), runs
+ * `steps` PIC steps (load interpolator, clear, advance_p per species
+ * [+ vpic_migrate_particles when the context exchanges or absorbs],
+ * unload [+ advance_b(1/2), advance_e, advance_b(1/2) if field_solve]) and
+ * downloads jf (nv x 4 floats) into jf_host and, if host_out, the particles.
+ * Period k+1's upload and period k-1's download run on internal copy streams
+ * under period k's compute (events order them).  deposit_modes (nullable):
+ * [steps][nsp] VPIC_OPT_DEPOSIT values per step and species (the caller's
+ * AUTO policy).  *pushes (host, nullable) = particles x PIC steps done.
+ * ENQUEUES on `stream` (which finally waits for the copy streams); host
+ * buffers must stay valid until `stream` is synchronised.  Synchronises only
+ * where vpic_migrate_particles does.  Errors: VPIC_ERR_INVALID (bad
+ * argument), VPIC_ERR_CAPACITY (workspace too small), or the error of the
+ * failing call (work already enqueued is left on the stream). */
+int vpic_run_host(vpic_ctx *ctx, int nsp, const vpic_species_host_t *sp, const float *fields_host,
+                  float *jf_host, int order, int64_t tile_sz, int steps, int n_cycles,
+                  const int8_t *deposit_modes, int field_solve, float eps0, void *ws, size_t ws_bytes,
+                  int64_t *pushes, void *stream);
+
 #ifdef __cplusplus
 }
 #endif

@@ -48,6 +48,7 @@ def _units():
         ("gather_scatter.o", "gather_scatter.cu", []),
         ("diagnostics.o", "diagnostics.cu", ["-fmad=false"]),
         ("abi.o", "abi.cu", []),
+        ("host_driver.o", "host_driver.cu", []),
     ], I
 
 

@@ -155,6 +155,8 @@ class HotPath:
                 sp.np_dev = torch.tensor([sp.np], dtype=torch.int64, device=self.dev)
         self._graphs = {}
         self._warm = False
+        self._host_bufs = None  # run_host_cycles: the 4 device buffers per species
+        self._host_ws = None
         self.adv_events = []   # (start, end) CUDA events around advance_p, when recording
         self.sort_events = []  # (start, end, species) around vpic_sort_particles
         self.record_advance = False
@@ -303,77 +305,32 @@ class HotPath:
 
     # ------------------------------------------------------- host <-> device --
     def run_host_cycles(self, host_in, host_out, fields_host, jf_host, n_cycles: int, S: int):
-        """Stream `n_cycles` sort periods from pinned host memory: every cycle
-        uploads its particle and field inputs and downloads jf and, unless
-        host_out is None, its particles.  The H2D of cycle k+1 and the D2H of cycle k run on copy streams
-        under the neighbouring cycles' compute; 4 device particle buffers per
-        species rotate through input / sort scratch / result / spare.
-        Returns the pushes done (particles x PIC steps)."""
-        comp = torch.cuda.current_stream()
-        h2d, d2h = torch.cuda.Stream(), torch.cuda.Stream()
-        nsp = len(self.species)
-        pool = [[s.p, s.scratch, torch.empty_like(s.p), torch.empty_like(s.p)] for s in self.species]
-        fbuf = [self.fields, torch.empty_like(self.fields)]
-        jstage = [torch.empty_like(self.jf), torch.empty_like(self.jf)]
-        free_ev = {}                      # (species, buffer) -> event after which it is reusable
-        ev_comp, ev_out = {}, {}          # per cycle: compute done, download done
-        IN, SC = [0] * nsp, [1] * nsp
-        SPARE = [[2, 3] for _ in range(nsp)]
-
-        def upload(k, bufs):
-            with torch.cuda.stream(h2d):
-                for j in range(nsp):
-                    ev = free_ev.pop((j, bufs[j]), None)
-                    if ev is not None:
-                        h2d.wait_event(ev)
-                    pool[j][bufs[j]][:host_in[j].shape[0]].copy_(host_in[j], non_blocking=True)
-                if k - 2 in ev_comp:
-                    h2d.wait_event(ev_comp[k - 2])  # cycle k-2 read these fields
-                fbuf[k % 2].copy_(fields_host, non_blocking=True)
-                ev = torch.cuda.Event()
-                ev.record(h2d)
-            return ev
-
-        ev_in = upload(0, IN)
-        pushes = 0
-        for k in range(n_cycles):
-            nxt, ev_next = None, None
-            if k + 1 < n_cycles:
-                nxt = [SPARE[j].pop(0) for j in range(nsp)]
-                ev_next = upload(k + 1, nxt)
-            comp.wait_event(ev_in)
-            for j, sp in enumerate(self.species):
-                sp.p, sp.scratch = pool[j][IN[j]], pool[j][SC[j]]
-                sp.np = host_in[j].shape[0]
-            self.fields = fbuf[k % 2]
-            self.cycle(S)
-            pushes += S * self.n_particles
-            if k - 2 in ev_out:
-                comp.wait_event(ev_out[k - 2])     # jf staging buffer downloaded
-            jstage[k % 2].copy_(self.jf, non_blocking=True)
-            ev_c = torch.cuda.Event()
-            ev_c.record(comp)
-            ev_comp[k] = ev_c
-            res = [next(b for b in (IN[j], SC[j]) if pool[j][b] is self.species[j].p)
-                   for j in range(nsp)]
-            with torch.cuda.stream(d2h):
-                d2h.wait_event(ev_c)
-                for j, sp in enumerate(self.species if host_out is not None else ()):
-                    n = min(sp.np, host_out[j].shape[0])
-                    host_out[j][:n].copy_(sp.p[:n], non_blocking=True)
-                jf_host.copy_(jstage[k % 2], non_blocking=True)
-                ev_o = torch.cuda.Event()
-                ev_o.record(d2h)
-            ev_out[k] = ev_o
-            for j in range(nsp):
-                free_ev[(j, res[j])] = ev_o
-                other = SC[j] if res[j] == IN[j] else IN[j]
-                SPARE[j].append(res[j])
-                if nxt is not None:
-                    IN[j], SC[j] = nxt[j], other
-            ev_in = ev_next
-        comp.wait_stream(d2h)
-        comp.wait_stream(h2d)
+        """Stream `n_cycles` sort periods from pinned host memory through the
+        C ABI's host-buffer driver (vpic_run_host): every cycle uploads its
+        particle and field inputs and downloads jf and, unless host_out is
+        None, its particles; the library overlaps cycle k+1's upload and
+        cycle k-1's download with cycle k's compute (4 device particle
+        buffers per species rotate).  The deposit mode per species and step
+        is this HotPath's (AUTO policy or fixed).  Returns the pushes done
+        (particles x PIC steps)."""
+        if self._host_bufs is None:
+            self._host_bufs = [[s.p, s.scratch, torch.empty_like(s.p), torch.empty_like(s.p)]
+                               for s in self.species]
+        species = [(s.q, s.m, host_in[j], None if host_out is None else host_out[j], host_in[j].shape[0],
+                    self._host_bufs[j]) for j, s in enumerate(self.species)]
+        modes = np.empty((S, len(self.species)), np.int8)
+        for t in range(S):
+            for j, sp in enumerate(self.wl.species):
+                modes[t, j] = (auto_deposit_mode(sp.u_th, self.g.cvac, self.g.dt,
+                                                 min(self.g.dx, self.g.dy, self.g.dz), t)
+                               if self.deposit_auto else self._dep_mode)
+        need = vpic.vpic_run_host_workspace_bytes(self.ctx, species, self.order)
+        if self._host_ws is None or self._host_ws.numel() < need:
+            self._host_ws = torch.empty(need, dtype=torch.uint8, device=self.dev)
+        pushes = vpic.vpic_run_host(self.ctx, species, fields_host, jf_host, self.order, self.tile_sz, S,
+                                    n_cycles, modes, self.field_solve, self.eps0, self._host_ws)
+        for j, s in enumerate(self.species):
+            s.np = host_in[j].shape[0]
         return pushes
 
     def particles_host(self, k: int) -> np.ndarray:

@@ -35,7 +35,8 @@ EXPORTS = ["vpic_get_unique_id", "vpic_ctx_create", "vpic_ctx_destroy", "vpic_ct
            "vpic_sort_particles", "vpic_load_interpolator", "vpic_clear_accumulator",
            "vpic_advance_p", "vpic_advance_p_dev", "vpic_unload_accumulator", "vpic_migrate_particles", "vpic_migrate_particles_dev",
            "vpic_kernel_launches", "vpic_advance_b", "vpic_advance_e", "vpic_gather_scatter",
-           "vpic_accumulate_rho", "vpic_continuity_residual"]
+           "vpic_accumulate_rho", "vpic_continuity_residual", "vpic_run_host_workspace_bytes",
+           "vpic_run_host"]
 
 
 class VpicError(RuntimeError):
@@ -88,6 +89,9 @@ def load(path: str = LIB_PATH) -> ctypes.CDLL:
                                     I64, P, I64, P, P, P], I),
         "vpic_advance_p_dev": ([P, ctypes.c_float, ctypes.c_float, P, P, I64, P, P, P, I64, P, P, P], I),
         "vpic_migrate_particles_dev": ([P, ctypes.c_float, ctypes.c_float, P, P, I64, P, I64, P, P, P, P], I),
+        "vpic_run_host_workspace_bytes": ([P, I, P, I], ctypes.c_size_t),
+        "vpic_run_host": ([P, I, P, P, P, I, I64, I, I, P, I, ctypes.c_float, P, ctypes.c_size_t,
+                           ctypes.POINTER(I64), P], I),
     }
     for name, (args, res) in sig.items():
         f = getattr(lib, name)
@@ -269,6 +273,52 @@ def vpic_migrate_particles_dev(ctx: Context, q: float, m: float, p, np_dev, max_
 
 
 # ------------------------------------------------------- tensor helpers --
+class vpic_species_host_t(ctypes.Structure):
+    _fields_ = [("q", ctypes.c_float), ("m", ctypes.c_float), ("host_in", ctypes.c_void_p),
+                ("host_out", ctypes.c_void_p), ("np", ctypes.c_int64), ("max_np", ctypes.c_int64),
+                ("dev", ctypes.c_void_p * 4)]
+
+
+def _species_host(species):
+    """[(q, m, host_in, host_out | None, np, [4 device buffers])] -> C array."""
+    arr = (vpic_species_host_t * len(species))()
+    for k, (q, m, hin, hout, n, dev) in enumerate(species):
+        assert hin.is_pinned() and (hout is None or hout.is_pinned()), "host buffers must be pinned"
+        arr[k].q, arr[k].m = q, m
+        arr[k].host_in = hin.data_ptr()
+        arr[k].host_out = hout.data_ptr() if hout is not None else None
+        arr[k].np = n
+        arr[k].max_np = min(b.shape[0] for b in dev)
+        for b in range(4):
+            arr[k].dev[b] = dev[b].data_ptr()
+    return arr
+
+
+def vpic_run_host_workspace_bytes(ctx: Context, species, order: int) -> int:
+    arr = _species_host(species)
+    return int(load().vpic_run_host_workspace_bytes(ctx.h, len(species), arr, order))
+
+
+def vpic_run_host(ctx: Context, species, fields_host, jf_host, order: int, tile_sz: int, steps: int,
+                  n_cycles: int, deposit_modes=None, field_solve: bool = False, eps0: float = 1.0,
+                  ws=None, stream=None) -> int:
+    """n_cycles sort periods from / to pinned host memory through the C ABI
+    (copies pipelined inside the library); returns particles x PIC steps."""
+    import numpy as np
+    arr = _species_host(species)
+    modes = None
+    if deposit_modes is not None:
+        modes = np.ascontiguousarray(deposit_modes, dtype=np.int8)
+        assert modes.size == steps * len(species)
+    pushes = ctypes.c_int64(0)
+    ws_bytes = 0 if ws is None else ws.numel() * ws.element_size()
+    _check("vpic_run_host", load().vpic_run_host(
+        ctx.h, len(species), arr, fields_host.data_ptr(), jf_host.data_ptr(), order, tile_sz, steps,
+        n_cycles, modes.ctypes.data if modes is not None else None, int(field_solve), eps0, _ptr(ws),
+        ws_bytes, ctypes.byref(pushes), _stream(stream)))
+    return int(pushes.value)
+
+
 def particles_to_device(p_np, device="cuda") -> torch.Tensor:
     """Host structured particle array -> device float32 [n, 8] view (32 B records)."""
     import numpy as np

@@ -438,7 +438,10 @@ def our_arm(args, rank, world):
 
         e2e = {"value": timed_e2e(None), "unit": UNIT, "h2d_bytes_per_step": h2d,
                "d2h_bytes_per_step": jf_host.numel() * 4,
-               "result": "jf (current density) read back every step"}
+               "result": "jf (current density) read back every step",
+               "api": "vpic_run_host (C ABI): particles + fields uploaded from pinned host memory and jf "
+                      "downloaded every step (one step = one sort period), copies pipelined on the "
+                      "library's copy streams"}
         if world == 1:   # (N > 1: 17 GB more pinned host memory per rank; skipped)
             host_out = [torch.empty(tuple(h.shape), dtype=torch.float32, pin_memory=True)
                         for h in host_in]

@@ -352,15 +352,13 @@ def to_global(gg: GridSpec, gb: GridSpec, p: np.ndarray) -> np.ndarray:
 
 
 def block_fields(gg: GridSpec, gb: GridSpec, f: np.ndarray) -> np.ndarray:
-    """fields[nv_block][8] of block gb cut from the global fields (interior and
-    ghost voxels; ghost coordinates wrap periodically on the global box)."""
+    """fields[nv_block][8] of block gb cut from the global fields: interior
+    and ghost voxels at the same global coordinates (a block's ghost plane is
+    the neighbour block's interior plane, or the global box's own ghost plane
+    on an outer face -- which a wall's caller-owned ghost values need)."""
     v = np.arange(gb.nv)
     x, y, z = gb.coords(v)
-    n = (gg.nx, gg.ny, gg.nz)
-    X = (x + gb.gx0 - 1) % n[0] + 1
-    Y = (y + gb.gy0 - 1) % n[1] + 1
-    Z = (z + gb.gz0 - 1) % n[2] + 1
-    return f[gg.voxel(X, Y, Z)].copy()
+    return f[gg.voxel(x + gb.gx0, y + gb.gy0, z + gb.gz0)].copy()
 
 
 def block_interior_to_global(gg: GridSpec, gb: GridSpec) -> Tuple[np.ndarray, np.ndarray]:

@@ -33,10 +33,23 @@ def global_workload():
 
 def main():
     out = sys.argv[1]
+    modes = MODES
     rank, world = int(os.environ["RANK"]), int(os.environ["WORLD_SIZE"])
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if os.environ.get("MR_ONE_GPU") == "1":
+        # every rank on GPU 0: NCCL refuses two ranks of one communicator on
+        # one device of one host, so each rank poses as its own host
+        # (NCCL_HOSTID) and the ranks talk through NCCL's socket transport on
+        # the loopback interface -- the real multi-rank NCCL send/recv code
+        # path of migrate.cu, without NVLink (so without the device-initiated
+        # modes, whose symmetric-memory peers must be NVLink-reachable)
+        local = 0
+        os.environ["NCCL_HOSTID"] = f"vpic-mr-{rank}"
+        os.environ.setdefault("NCCL_SOCKET_IFNAME", "lo")
+        os.environ.setdefault("NCCL_IB_DISABLE", "1")
+        modes = [m for m in MODES if m[0] == "nccl"]
     torch.cuda.set_device(local)
-    dist.init_process_group("nccl")
+    dist.init_process_group("gloo" if os.environ.get("MR_ONE_GPU") == "1" else "nccl")
     wl = global_workload()
     gg = wl.grid
     gb = inputs.strong_decompose(gg, world, rank)
@@ -46,7 +59,7 @@ def main():
     wlb = replace(wl, grid=gb)
     vb, vg = inputs.block_interior_to_global(gg, gb)
     res = {}
-    for exch, mig in MODES:
+    for exch, mig in modes:
         obj = [vpic.vpic_get_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
         hp = HotPath(wlb, parts, fields, math=vpic.MATH_IEEE, rank=rank, nranks=world, uid=obj[0],

@@ -446,6 +446,10 @@ def test_block_split_roundtrip(nranks):
         fb = inputs.block_fields(gg, gb, f)
         vb, vg = inputs.block_interior_to_global(gg, gb)
         assert np.array_equal(fb[vb], f[vg])
+        # every block voxel, ghosts included, holds the global value at its
+        # global coordinates (outer-face ghost planes are the box's own)
+        x, y, z = gb.coords(np.arange(gb.nv))
+        assert np.array_equal(fb, f[gg.voxel(x + gb.gx0, y + gb.gy0, z + gb.gz0)])
         cover[vg] += 1
     key = lambda a: np.sort(np.ascontiguousarray(a).view(np.dtype((np.void, 32))))
     assert np.array_equal(key(np.concatenate(back)), key(p))

@@ -32,6 +32,10 @@ sys.path.insert(0, ROOT)
 import numpy as np  # noqa: E402
 
 FALLBACK_HBM_GBS = 6650.0
+# VPIC_BENCH_SHARE_GPU=1 (test of the N > 1 code path on a 1-GPU box, not a
+# measurement): every rank on GPU 0, torch.distributed over gloo, and the
+# library's NCCL communicator over sockets (each rank poses as its own host)
+SHARE_GPU = os.environ.get("VPIC_BENCH_SHARE_GPU") == "1"
 METRIC = "particle pushes/sec (advance_p+sort)"
 UNIT = "pushes/s"
 
@@ -288,9 +292,10 @@ def our_arm(args, rank, world):
     from paper_conf_sc_tanlta25_b200.pic import HotPath
 
     from paper_conf_sc_tanlta25_b200.pic import bind_to_gpu_cpus
-    local = int(os.environ.get("LOCAL_RANK", "0"))
+    local = 0 if SHARE_GPU else int(os.environ.get("LOCAL_RANK", "0"))
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
+    red_dev = "cpu" if SHARE_GPU else dev   # gloo reduces host tensors
     # pinned e2e buffers first-touched on the GPU's NUMA node (2-socket nodes)
     cpu_bind = bind_to_gpu_cpus(local)
     # N > 1: weak scaling on configs[3] (C2 per GPU), or strong scaling of
@@ -396,7 +401,7 @@ def our_arm(args, rank, world):
     sort_ms = {k: round(sum(v) / len(v), 3) for k, v in sort_ms.items()}
     adv_np = sum(n for _, n in adv) / len(adv)
     t = torch.tensor([ms, float(pushes_local), float(n_local), float(hp.n_particles)],
-                     dtype=torch.float64, device=dev)
+                     dtype=torch.float64, device=red_dev)
     if world > 1:
         tmax = t.clone()
         dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
@@ -430,7 +435,7 @@ def our_arm(args, rank, world):
             a1.record(stream)
             torch.cuda.synchronize()
             barrier()
-            t = torch.tensor([a0.elapsed_time(a1), float(n)], dtype=torch.float64, device=dev)
+            t = torch.tensor([a0.elapsed_time(a1), float(n)], dtype=torch.float64, device=red_dev)
             if world > 1:
                 tm = t.clone(); dist.all_reduce(tm, op=dist.ReduceOp.MAX)
                 ts = t.clone(); dist.all_reduce(ts, op=dist.ReduceOp.SUM)
@@ -524,7 +529,7 @@ def spawn_ranks(n: int) -> int:
     import socket
     import torch
     have = torch.cuda.device_count()
-    if have < n:
+    if have < n and not SHARE_GPU:
         print(f"bench.py: --gpus {n} but {have} GPU(s) visible", file=sys.stderr, flush=True)
         return 2
     with socket.socket() as s:
@@ -548,8 +553,12 @@ def main():
     if world > 1:
         import torch
         import torch.distributed as dist
-        torch.cuda.set_device(int(os.environ.get("LOCAL_RANK", "0")))
-        dist.init_process_group("nccl")
+        if SHARE_GPU:
+            os.environ["NCCL_HOSTID"] = f"vpic-bench-{rank}"
+            os.environ.setdefault("NCCL_SOCKET_IFNAME", "lo")
+            os.environ.setdefault("NCCL_IB_DISABLE", "1")
+        torch.cuda.set_device(0 if SHARE_GPU else int(os.environ.get("LOCAL_RANK", "0")))
+        dist.init_process_group("gloo" if SHARE_GPU else "nccl")
         if rank == 0:
             print(f"bench.py: NCCL process group initialised, nranks={dist.get_world_size()}",
                   file=sys.stderr, flush=True)

@@ -81,3 +81,25 @@ def test_multirank_exchange_matches_oracle(orc, tmp_path):
     sys.path.insert(0, HERE)
     import multirank_worker as W
     _run_and_compare(orc, tmp_path, nranks, {}, W.MODES)
+
+
+@pytest.mark.timeout(900)
+def test_bench_multirank_path_on_one_gpu():
+    """bench.py's N > 1 path end to end (self-launch of the ranks, process
+    grid, NCCL communicator, migration, max-over-ranks timing, the global
+    conservation check, the C-ABI e2e leg) with 2 ranks sharing GPU 0
+    (VPIC_BENCH_SHARE_GPU: gloo for torch.distributed, the library's NCCL
+    over sockets; a functional test, not a measurement), on the f3 strong-
+    scaling box."""
+    import json
+    env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK")}
+    env["VPIC_BENCH_SHARE_GPU"] = "1"
+    r = subprocess.run([sys.executable, os.path.join(os.path.dirname(HERE), "bench.py"), "--gpus", "2",
+                        "--config", "5", "--steps", "1", "--warmup", "1", "--no-cpu-baseline",
+                        "--exchange", "nccl"], capture_output=True, text=True, env=env, timeout=800)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-3000:]
+    line = json.loads(r.stdout.strip().splitlines()[-1])
+    assert line["n_gpus"] == 2 and line["scaling"] == "strong"
+    assert line["comm"]["nranks"] == 2 and line["comm"]["vpic_ctx_nranks"] == 2
+    assert line["conservation"]["ok"]
+    assert line["e2e"]["value"] > 0

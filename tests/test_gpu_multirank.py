@@ -29,7 +29,18 @@ def _ngpu():
     return torch.cuda.device_count() if torch.cuda.is_available() else 0
 
 
+def _free_gpu_memory():
+    """The subprocesses need the GPU memory this pytest process may still
+    cache from earlier (full-size) tests."""
+    import gc
+    gc.collect()
+    if torch.cuda.is_available():
+        torch.cuda.synchronize()
+        torch.cuda.empty_cache()
+
+
 def _run_and_compare(orc, tmp_path, nranks, env_extra, modes):
+    _free_gpu_memory()
     import multirank_worker as W
     from paper_conf_sc_tanlta25_b200 import _build
     from paper_conf_sc_tanlta25_b200 import inputs
@@ -92,6 +103,7 @@ def test_bench_multirank_path_on_one_gpu():
     over sockets; a functional test, not a measurement), on the f3 strong-
     scaling box."""
     import json
+    _free_gpu_memory()
     env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK")}
     env["VPIC_BENCH_SHARE_GPU"] = "1"
     r = subprocess.run([sys.executable, os.path.join(os.path.dirname(HERE), "bench.py"), "--gpus", "2",

@@ -188,6 +188,17 @@ int vpic_sort_particles(vpic_ctx *ctx, const vpic_particle_t *p_in, vpic_particl
                         int32_t *voxel_counts, int64_t *new_keys, int64_t *perm,
                         void *stream);
 
+/* vpic_sort_particles with the voxel key of every input particle supplied
+ * (keys[np] uint32 device, 4-B aligned -- e.g. written by the last
+ * vpic_advance_p_keys of a sort period), so the sort does not read a 32-B
+ * sector of every record to get its 4-B key (SURVEY.md §8(a) a1 fused into
+ * the push).  keys[i] must equal p_in[i].i; otherwise identical to
+ * vpic_sort_particles (outputs, workspace, errors, enqueue-only). */
+int vpic_sort_particles_keyed(vpic_ctx *ctx, const vpic_particle_t *p_in, vpic_particle_t *p_out,
+                              int64_t np, int order, int64_t tile_sz, const uint32_t *keys, void *ws,
+                              size_t ws_bytes, int32_t *voxel_counts, int64_t *new_keys,
+                              int64_t *perm, void *stream);
+
 /* ---------------------------------------------------- (a5) interpolator -- */
 
 /* Fill the +x/+y/+z ghost planes of fields (locally periodic faces: copy of
@@ -219,6 +230,16 @@ int vpic_clear_accumulator(vpic_ctx *ctx, float *acc, void *stream);
 int vpic_advance_p(vpic_ctx *ctx, float q, float m, vpic_particle_t *p, int64_t np,
                    const float *interp, float *acc, vpic_mover_t *movers, int64_t max_movers,
                    int64_t *n_movers, int32_t *flags, void *stream);
+
+/* vpic_advance_p that also writes keys_out[i] = p[i].i as the call leaves
+ * particle i (keys_out[np] uint32 device, 4-B aligned): the keys of the next
+ * vpic_sort_particles_keyed, at the cost of a coalesced 4-B store per
+ * particle.  Valid for that sort only if the call produced no movers (a
+ * mover's record holds its stop code and vpic_migrate_particles reorders the
+ * array). */
+int vpic_advance_p_keys(vpic_ctx *ctx, float q, float m, vpic_particle_t *p, int64_t np,
+                        const float *interp, float *acc, vpic_mover_t *movers, int64_t max_movers,
+                        int64_t *n_movers, int32_t *flags, uint32_t *keys_out, void *stream);
 
 /* Same, with the particle count in DEVICE memory (*np_dev, int64, 8-byte
  * aligned; read by the kernels at run time, min(*np_dev, max_np) particles are

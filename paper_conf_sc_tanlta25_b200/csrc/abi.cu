@@ -60,12 +60,12 @@ void note_launch(int n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
 cudaError_t launch_advance_p(const vpic_ctx *c, float qsp, float msp, vpic_particle_t *p,
                              int64_t np, const float *interp, float *acc, vpic_mover_t *movers,
                              int64_t max_movers, int64_t *n_movers, int32_t *flags,
-                             cudaStream_t s, const int64_t *np_dev) {
+                             cudaStream_t s, const int64_t *np_dev, uint32_t *keys_out) {
   if (c->math == MATH_IEEE)
     return launch_advance_p_ieee(c, qsp, msp, p, np, interp, acc, movers, max_movers, n_movers,
-                                 flags, s, np_dev);
+                                 flags, s, np_dev, keys_out);
   return launch_advance_p_fast(c, qsp, msp, p, np, interp, acc, movers, max_movers, n_movers,
-                               flags, s, np_dev);
+                               flags, s, np_dev, keys_out);
 }
 }  // namespace vpic
 
@@ -258,6 +258,26 @@ int vpic_sort_particles(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_
                                  new_keys, perm, S(stream)));
 }
 
+int vpic_sort_particles_keyed(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_t *p_out,
+                              int64_t np, int order, int64_t tile_sz, const uint32_t *keys, void *ws,
+                              size_t ws_bytes, int32_t *voxel_counts, int64_t *new_keys, int64_t *perm,
+                              void *stream) {
+  VPIC_NVTX();
+  if (!c || np < 0 || np >= ((int64_t)1 << 32) || order < 0 || order > 3 || tile_sz < 0)
+    return VPIC_ERR_INVALID;
+  if (np > 0 && (!p_in || !p_out || !keys || !aligned16(p_in) || !aligned16(p_out) ||
+                 (reinterpret_cast<uintptr_t>(keys) & 3u)))
+    return VPIC_ERR_INVALID;
+  if (np > 0 && p_in == p_out) return VPIC_ERR_INVALID;
+  if (np > 0 && order != VPIC_SORT_NONE) {
+    if (!ws) return VPIC_ERR_INVALID;
+    if (ws_bytes < sort_workspace_bytes(c, np, order)) return VPIC_ERR_CAPACITY;
+  }
+  DeviceGuard dg(c->device);
+  return cuda_status(launch_sort(c, p_in, p_out, np, order, tile_sz, ws, ws_bytes, voxel_counts,
+                                 new_keys, perm, S(stream), keys));
+}
+
 int vpic_load_interpolator(vpic_ctx *c, float *fields, float *interp, void *stream) {
   VPIC_NVTX();
   if (!c || !fields || !interp || !aligned16(fields) || !aligned32(interp)) return VPIC_ERR_INVALID;
@@ -291,6 +311,22 @@ int vpic_advance_p(vpic_ctx *c, float q, float m, vpic_particle_t *p, int64_t np
   DeviceGuard dg(c->device);
   return cuda_status(launch_advance_p(c, q, m, p, np, interp, acc, movers, max_movers, n_movers,
                                       flags, S(stream)));
+}
+
+int vpic_advance_p_keys(vpic_ctx *c, float q, float m, vpic_particle_t *p, int64_t np,
+                        const float *interp, float *acc, vpic_mover_t *movers, int64_t max_movers,
+                        int64_t *n_movers, int32_t *flags, uint32_t *keys_out, void *stream) {
+  VPIC_NVTX();
+  if (!c || np < 0 || np >= ((int64_t)1 << 31) || !(m > 0) || max_movers < 0) return VPIC_ERR_INVALID;
+  if (np == 0) return VPIC_OK;
+  if (!p || !interp || !acc || !n_movers || !keys_out || !aligned16(p) || !aligned32(interp) ||
+      !aligned16(acc) || (reinterpret_cast<uintptr_t>(keys_out) & 3u))
+    return VPIC_ERR_INVALID;
+  if (max_movers > 0 && (!movers || !aligned16(movers))) return VPIC_ERR_INVALID;
+  if ((reinterpret_cast<uintptr_t>(n_movers) & 7u) != 0) return VPIC_ERR_INVALID;
+  DeviceGuard dg(c->device);
+  return cuda_status(launch_advance_p(c, q, m, p, np, interp, acc, movers, max_movers, n_movers,
+                                      flags, S(stream), nullptr, keys_out));
 }
 
 int vpic_advance_p_dev(vpic_ctx *c, float q, float m, vpic_particle_t *p, const int64_t *np_dev,

@@ -111,6 +111,32 @@ k_keys_count(const vpic_particle_t *__restrict__ p, int64_t n, uint32_t *__restr
   }
 }
 
+// The same from keys supplied by the caller (vpic_sort_particles_keyed:
+// written by the last advance_p): a coalesced 4-B read per particle instead
+// of a 32-B sector of its record.
+__global__ void __launch_bounds__(256)
+k_count_keys(const uint32_t *__restrict__ keys_in, int64_t n, uint32_t *__restrict__ count,
+             int64_t *__restrict__ new_keys) {
+  const int lane = threadIdx.x & 31;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t base = (int64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31); base < n;
+       base += stride) {
+    const int64_t i = base + lane;
+    const bool valid = i < n;
+    uint32_t k = 0xffffffffu;
+    if (valid) {
+      k = __ldcs(keys_in + i);
+      if (new_keys) new_keys[i] = (int64_t)k;
+    }
+    const uint32_t prev = __shfl_up_sync(FULL, k, 1);
+    const bool head = valid && (lane == 0 || prev != k);
+    const unsigned ends = __ballot_sync(FULL, head) | ~__ballot_sync(FULL, valid);
+    const unsigned above = lane == 31 ? 0u : (ends & ~((2u << lane) - 1u));
+    const int len = (above ? __ffs(above) - 1 : 32) - lane;
+    if (head) atomicAdd(&count[k], (uint32_t)len);
+  }
+}
+
 // Digit histograms of every LSD pass from the voxel histogram.
 __global__ void k_digit_hist(const uint32_t *__restrict__ count, int64_t nv, PassDesc pd,
                              uint32_t *__restrict__ ghist) {
@@ -670,19 +696,21 @@ template <class KeyT>
 cudaError_t lsd_sort(const PassDesc &pd, int64_t n, KeyT *kA, KeyT *kB, uint32_t *vA,
                      uint32_t *vB, const uint32_t *vals0, uint32_t *ghist, uint32_t *goff,
                      unsigned long long *status, unsigned int *ctr, bool need_keys_out,
-                     const int *live_bits, KeyT **k_final, uint32_t **v_final, cudaStream_t s) {
+                     const int *live_bits, KeyT **k_final, uint32_t **v_final, cudaStream_t s,
+                     const KeyT *k_first = nullptr /* the first pass's keys, if not in kA */) {
   CK(cudaMemsetAsync(ctr, 0, 4 * MAX_PASSES, s));
   k_scan_hist<<<pd.npass, 256, 0, s>>>(ghist, goff, pd); note_launch();
   CK(cudaGetLastError());
   const int64_t tiles = (n + TILE - 1) / TILE;
   KeyT *kin = kA, *kout = kB;
+  const KeyT *kin0 = k_first ? k_first : kA;
   const uint32_t *vin = vals0;
   uint32_t *vout = (vals0 == vA) ? vB : vA;
   for (int q = 0; q < pd.npass; ++q) {
     CK(cudaMemsetAsync(status, 0, 8 * (size_t)tiles * (1 << pd.bits[q]), s));
     const bool last = q == pd.npass - 1;
-    CK(radix_pass<KeyT>(pd.bits[q], kin, vin, (last && !need_keys_out) ? nullptr : kout, vout, n,
-                        pd.shift[q], goff + q * (1 << MAX_BITS), status, ctr + q, live_bits, s));
+    CK(radix_pass<KeyT>(pd.bits[q], q == 0 ? kin0 : kin, vin, (last && !need_keys_out) ? nullptr : kout,
+                        vout, n, pd.shift[q], goff + q * (1 << MAX_BITS), status, ctr + q, live_bits, s));
     *k_final = kout;
     *v_final = vout;
     std::swap(kin, kout);
@@ -744,7 +772,8 @@ size_t sort_workspace_bytes(const vpic_ctx *c, int64_t np, int order) {
 
 cudaError_t launch_sort(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_t *p_out,
                         int64_t np, int order, int64_t tile_sz, void *ws, size_t ws_bytes,
-                        int32_t *voxel_counts, int64_t *new_keys, int64_t *perm, cudaStream_t s) {
+                        int32_t *voxel_counts, int64_t *new_keys, int64_t *perm, cudaStream_t s,
+                        const uint32_t *keys_in) {
   const int64_t nv = c->gk.nv;
   const int sms = c->num_sms;
   if (np == 0) {
@@ -783,8 +812,13 @@ cudaError_t launch_sort(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_
   uint32_t *count = voxel_counts ? reinterpret_cast<uint32_t *>(voxel_counts)
                                  : reinterpret_cast<uint32_t *>(w + L.count);
   CK(cudaMemsetAsync(count, 0, 4 * (size_t)nv, s));
-  k_keys_count<<<grid_cap(np, 256, sms, 8), 256, 0, s>>>(
-      p_in, np, kA, count, (order == VPIC_SORT_STANDARD) ? new_keys : nullptr); note_launch();
+  if (keys_in) {   // keys from the caller: histogram only (the first pass reads keys_in)
+    k_count_keys<<<grid_cap(np, 256, sms, 8), 256, 0, s>>>(
+        keys_in, np, count, (order == VPIC_SORT_STANDARD) ? new_keys : nullptr); note_launch();
+  } else {
+    k_keys_count<<<grid_cap(np, 256, sms, 8), 256, 0, s>>>(
+        p_in, np, kA, count, (order == VPIC_SORT_STANDARD) ? new_keys : nullptr); note_launch();
+  }
   CK(cudaGetLastError());
   const PassDesc pd = make_passes(bits_for((uint64_t)(nv - 1)));
   CK(cudaMemsetAsync(ghist, 0, 4 * (size_t)MAX_PASSES * (1 << MAX_BITS), s));
@@ -794,7 +828,7 @@ cudaError_t launch_sort(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_
   uint32_t *K = nullptr, *P = nullptr;
   const bool need_offs = order != VPIC_SORT_STANDARD;
   CK(lsd_sort<uint32_t>(pd, np, kA, kB, vA, vB, nullptr, ghist, goff, status, ctr, need_offs,
-                        nullptr, &K, &P, s));
+                        nullptr, &K, &P, s, keys_in));
   const RankParams *sel = nullptr;
   uint32_t *P_alt = nullptr;
   if (need_offs) {  // offs[k] = first standard position of voxel k; max_r

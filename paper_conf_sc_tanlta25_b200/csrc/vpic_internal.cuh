@@ -40,6 +40,9 @@ struct GridK {
   // 9(oz+1), o = -1 / 0 / +1 for ghost coordinate 0 / interior / n+1
   int32_t ghost_mig;
   unsigned char *di_peer26[27];  // device-initiated: inbox of the direction-d neighbour
+  // vpic_advance_p_keys: every particle's voxel after the move, for the next
+  // sort (null otherwise; set per launch)
+  uint32_t *keys_out;
 };
 
 // Round-up reciprocal for exact unsigned division of n < 2^31 by d >= 2:
@@ -131,16 +134,19 @@ inline void once_per_device(std::atomic<uint64_t> &done, F &&f) {
 cudaError_t launch_advance_p(const vpic_ctx *c, float qsp, float msp, vpic_particle_t *p,
                              int64_t np, const float *interp, float *acc, vpic_mover_t *movers,
                              int64_t max_movers, int64_t *n_movers, int32_t *flags,
-                             cudaStream_t s, const int64_t *np_dev = nullptr);
+                             cudaStream_t s, const int64_t *np_dev = nullptr,
+                             uint32_t *keys_out = nullptr);
 // the two math variants are compiled from the same source (advance_p.cu)
 cudaError_t launch_advance_p_fast(const vpic_ctx *c, float qsp, float msp, vpic_particle_t *p,
                                   int64_t np, const float *interp, float *acc,
                                   vpic_mover_t *movers, int64_t max_movers, int64_t *n_movers,
-                                  int32_t *flags, cudaStream_t s, const int64_t *np_dev = nullptr);
+                                  int32_t *flags, cudaStream_t s, const int64_t *np_dev = nullptr,
+                                  uint32_t *keys_out = nullptr);
 cudaError_t launch_advance_p_ieee(const vpic_ctx *c, float qsp, float msp, vpic_particle_t *p,
                                   int64_t np, const float *interp, float *acc,
                                   vpic_mover_t *movers, int64_t max_movers, int64_t *n_movers,
-                                  int32_t *flags, cudaStream_t s, const int64_t *np_dev = nullptr);
+                                  int32_t *flags, cudaStream_t s, const int64_t *np_dev = nullptr,
+                                  uint32_t *keys_out = nullptr);
 // move_p of a list of movers (incoming particles after migration)
 // n_in_dev (nullable): device count, n_in then only bounds it; di_round: the
 // migration round of the departures (device-initiated exchange only)
@@ -173,10 +179,12 @@ cudaError_t launch_gather_scatter(const vpic_ctx *c, const int32_t *keys, const 
                                   int64_t nkeys, int64_t nx, int aggregate, cudaStream_t s);
 
 size_t sort_workspace_bytes(const vpic_ctx *c, int64_t np, int order);
+// keys_in (nullable): the voxel of every input particle, supplied by the
+// caller (vpic_advance_p_keys) instead of read from the records
 cudaError_t launch_sort(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_t *p_out,
                         int64_t np, int order, int64_t tile_sz, void *ws, size_t ws_bytes,
                         int32_t *voxel_counts, int64_t *new_keys, int64_t *perm,
-                        cudaStream_t s);
+                        cudaStream_t s, const uint32_t *keys_in = nullptr);
 
 int migrate(vpic_ctx *c, float qsp, float msp, vpic_particle_t *p, int64_t *np, int64_t max_np,
             vpic_mover_t *movers, int64_t max_movers, const int64_t *n_movers, float *acc,

@@ -59,6 +59,8 @@ class SpeciesState:
     n_movers: torch.Tensor   # int64[1]
     flags: torch.Tensor      # int32[1]
     np_dev: torch.Tensor = None   # int64[1]: the count on the device (graph mode)
+    keys: torch.Tensor = None     # uint32-as-int32 [cap]: voxels from the last advance (keyed sort)
+    keys_valid: bool = False
 
 
 # thermal spread (cells) since the sort within which DEP_SMEM pays (DESIGN.md
@@ -83,7 +85,7 @@ class HotPath:
                  device: Optional[int] = None, field_solve: bool = False, eps0: float = 1.0,
                  loopback_exchange: bool = False, concurrent_species: bool = False,
                  device_exchange: bool = False, inbox_cap: int = 0, single_round: bool = False,
-                 graphs: bool = False):
+                 graphs: bool = False, keyed_sort: bool = True):
         vpic.load()
         self.wl = wl
         self.g = wl.grid
@@ -146,6 +148,7 @@ class HotPath:
         # synchronisation inside a period).  Needs no migration, or the
         # single-round device-initiated exchange.
         self.graphs = graphs
+        self.keyed_sort = keyed_sort    # the period's last push writes the next sort's keys
         if graphs:
             if self.migrate and not (single_round and device_exchange):
                 raise ValueError("graphs need the single-round device-initiated exchange (or none)")
@@ -186,16 +189,26 @@ class HotPath:
             if self.record_advance:
                 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 e0.record(stream)
-            vpic.vpic_sort_particles(self.ctx, s.p, s.scratch, s.np, order, self.tile_sz, self.ws)
+            if s.keys_valid:   # keys written by the period's last advance_p
+                vpic.vpic_sort_particles_keyed(self.ctx, s.p, s.scratch, s.np, order, self.tile_sz, s.keys,
+                                               self.ws)
+            else:
+                vpic.vpic_sort_particles(self.ctx, s.p, s.scratch, s.np, order, self.tile_sz, self.ws)
+            s.keys_valid = False
             if self.record_advance:
                 e1.record(stream)
                 self.sort_events.append((e0, e1, s.name))
             s.p, s.scratch = s.scratch, s.p
         self.steps_since_sort = 0
 
-    def step(self, do_sort: bool = False):
+    def step(self, do_sort: bool = False, emit_keys: bool = False):
+        """One PIC step.  emit_keys: the last step of a sort period -- the
+        push also writes every particle's voxel for the next sort
+        (vpic_advance_p_keys + vpic_sort_particles_keyed: no pass over the
+        records to read the keys), when nothing migrates."""
         if do_sort:
             self.sort()
+        keyed = emit_keys and self.keyed_sort and not self.migrate and not self.concurrent
         vpic.vpic_load_interpolator(self.ctx, self.fields, self.interp)
         vpic.vpic_clear_accumulator(self.ctx, self.acc)
         stream = torch.cuda.current_stream()
@@ -210,6 +223,7 @@ class HotPath:
                     e0.record(st)
                 vpic.vpic_advance_p(self.ctx, s.q, s.m, s.p, s.np, self.interp, self.acc, s.movers,
                                     s.movers.shape[0], s.n_movers, s.flags, stream=st)
+                s.keys_valid = False
                 if self.record_advance:
                     e1.record(st)
                     self.adv_events.append((e0, e1, s.np))
@@ -220,8 +234,15 @@ class HotPath:
             if self.record_advance:
                 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 e0.record(stream)
-            vpic.vpic_advance_p(self.ctx, s.q, s.m, s.p, s.np, self.interp, self.acc, s.movers,
-                                s.movers.shape[0], s.n_movers, s.flags)
+            if keyed:
+                if s.keys is None:
+                    s.keys = torch.empty(s.p.shape[0], dtype=torch.int32, device=self.dev)
+                vpic.vpic_advance_p_keys(self.ctx, s.q, s.m, s.p, s.np, self.interp, self.acc, s.movers,
+                                         s.movers.shape[0], s.n_movers, s.flags, s.keys)
+            else:
+                vpic.vpic_advance_p(self.ctx, s.q, s.m, s.p, s.np, self.interp, self.acc, s.movers,
+                                    s.movers.shape[0], s.n_movers, s.flags)
+            s.keys_valid = keyed
             if self.record_advance:
                 e1.record(stream)
                 self.adv_events.append((e0, e1, s.np))
@@ -245,7 +266,7 @@ class HotPath:
         if self.graphs:
             return self._cycle_graph(steps)
         for k in range(steps):
-            self.step(do_sort=(k == 0))
+            self.step(do_sort=(k == 0), emit_keys=(k == steps - 1))
 
     # ------------------------------------------------------- graph mode --
     def sync_counts(self):
@@ -267,6 +288,7 @@ class HotPath:
             self._set_deposit(k)
             vpic.vpic_advance_p_dev(self.ctx, s.q, s.m, s.p, s.np_dev, s.p.shape[0], self.interp, self.acc,
                                     s.movers, s.movers.shape[0], s.n_movers, s.flags)
+            s.keys_valid = False
             if self.migrate:
                 vpic.vpic_migrate_particles_dev(self.ctx, s.q, s.m, s.p, s.np_dev, s.p.shape[0], s.movers,
                                                 s.movers.shape[0], s.n_movers, self.acc, s.flags)
@@ -331,6 +353,7 @@ class HotPath:
                                     n_cycles, modes, self.field_solve, self.eps0, self._host_ws)
         for j, s in enumerate(self.species):
             s.np = host_in[j].shape[0]
+            s.keys_valid = False
         return pushes
 
     def particles_host(self, k: int) -> np.ndarray:

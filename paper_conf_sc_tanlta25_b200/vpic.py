@@ -36,7 +36,7 @@ EXPORTS = ["vpic_get_unique_id", "vpic_ctx_create", "vpic_ctx_destroy", "vpic_ct
            "vpic_advance_p", "vpic_advance_p_dev", "vpic_unload_accumulator", "vpic_migrate_particles", "vpic_migrate_particles_dev",
            "vpic_kernel_launches", "vpic_advance_b", "vpic_advance_e", "vpic_gather_scatter",
            "vpic_accumulate_rho", "vpic_continuity_residual", "vpic_run_host_workspace_bytes",
-           "vpic_run_host"]
+           "vpic_run_host", "vpic_sort_particles_keyed", "vpic_advance_p_keys"]
 
 
 class VpicError(RuntimeError):
@@ -90,6 +90,8 @@ def load(path: str = LIB_PATH) -> ctypes.CDLL:
         "vpic_advance_p_dev": ([P, ctypes.c_float, ctypes.c_float, P, P, I64, P, P, P, I64, P, P, P], I),
         "vpic_migrate_particles_dev": ([P, ctypes.c_float, ctypes.c_float, P, P, I64, P, I64, P, P, P, P], I),
         "vpic_run_host_workspace_bytes": ([P, I, P, I], ctypes.c_size_t),
+        "vpic_sort_particles_keyed": ([P, P, P, I64, I, I64, P, P, ctypes.c_size_t, P, P, P, P], I),
+        "vpic_advance_p_keys": ([P, ctypes.c_float, ctypes.c_float, P, I64, P, P, P, I64, P, P, P, P], I),
         "vpic_run_host": ([P, I, P, P, P, I, I64, I, I, P, I, ctypes.c_float, P, ctypes.c_size_t,
                            ctypes.POINTER(I64), P], I),
     }
@@ -196,6 +198,21 @@ def vpic_sort_particles(ctx: Context, p_in, p_out, np_: int, order: int, tile_sz
     _check("vpic_sort_particles", load().vpic_sort_particles(
         ctx.h, _ptr(p_in), _ptr(p_out), np_, order, tile_sz, _ptr(ws), ws_bytes,
         _ptr(voxel_counts), _ptr(new_keys), _ptr(perm), _stream(stream)))
+
+
+def vpic_sort_particles_keyed(ctx: Context, p_in, p_out, np_: int, order: int, tile_sz: int, keys,
+                              ws=None, voxel_counts=None, new_keys=None, perm=None, stream=None):
+    ws_bytes = 0 if ws is None else ws.numel() * ws.element_size()
+    _check("vpic_sort_particles_keyed", load().vpic_sort_particles_keyed(
+        ctx.h, _ptr(p_in), _ptr(p_out), np_, order, tile_sz, _ptr(keys), _ptr(ws), ws_bytes,
+        _ptr(voxel_counts), _ptr(new_keys), _ptr(perm), _stream(stream)))
+
+
+def vpic_advance_p_keys(ctx: Context, q: float, m: float, p, np_: int, interp, acc, movers=None,
+                        max_movers: int = 0, n_movers=None, flags=None, keys_out=None, stream=None):
+    _check("vpic_advance_p_keys", load().vpic_advance_p_keys(
+        ctx.h, q, m, _ptr(p), np_, _ptr(interp), _ptr(acc), _ptr(movers), max_movers,
+        _ptr(n_movers), _ptr(flags), _ptr(keys_out), _stream(stream)))
 
 
 def vpic_load_interpolator(ctx: Context, fields, interp, stream=None):

@@ -541,3 +541,61 @@ def test_sort_captures_in_cuda_graph(V, orc, order):
         assert np.array_equal(counts.cpu().numpy(), c_o)
         assert np.array_equal(nk.cpu().numpy(), nk_o)
         assert np.array_equal(perm.cpu().numpy(), perm_o)
+
+
+@pytest.mark.parametrize("order", [0, 1, 2], ids=["standard", "strided", "tiled"])
+def test_keyed_sort_matches_sort(V, orc, order):
+    """vpic_advance_p_keys writes every particle's voxel after its move (in-cell
+    items in the chunk, crossers after the drain); vpic_sort_particles_keyed
+    on those keys gives exactly the oracle's sort of the advanced particles
+    (hot particles: many crossers; ragged size; both kernels)."""
+    g = inputs.GridSpec(12, 9, 7)
+    p = inputs.random_particles(g, 40001, 81, u_scale=0.7)
+    f = inputs.make_fields(g, 0.05, seed=6)
+    for kernel in (1, 2):
+        ctx = mkctx(V, g, V.MATH_IEEE, 2, kernel)
+        fd = torch.from_numpy(f.copy()).cuda()
+        interp = torch.zeros((g.nv, 24), dtype=torch.float32, device="cuda")
+        V.vpic_load_interpolator(ctx, fd, interp)
+        acc = torch.zeros((g.nv, 12), dtype=torch.float32, device="cuda")
+        pd = dev_particles(V, p)
+        nm = torch.zeros(1, dtype=torch.int64, device="cuda")
+        keys = torch.full((p.size,), -5, dtype=torch.int32, device="cuda")
+        V.vpic_advance_p_keys(ctx, -1.0, 1.0, pd, p.size, interp, acc, None, 0, nm, None, keys)
+        torch.cuda.synchronize()
+        assert int(nm.item()) == 0
+        adv = V.particles_to_host(pd)
+        assert np.array_equal(keys.cpu().numpy(), adv["i"])
+        T = 29
+        out = torch.empty_like(pd)
+        ws = torch.empty(V.vpic_sort_workspace_bytes(ctx, p.size, order), dtype=torch.uint8, device="cuda")
+        counts = torch.empty(g.nv, dtype=torch.int32, device="cuda")
+        nk = torch.empty(p.size, dtype=torch.int64, device="cuda")
+        perm = torch.empty(p.size, dtype=torch.int64, device="cuda")
+        V.vpic_sort_particles_keyed(ctx, pd, out, p.size, order, T, keys, ws, counts, nk, perm)
+        torch.cuda.synchronize()
+        p_o, c_o, nk_o, perm_o = orc.sort_particles(g, adv, order, T)
+        assert_particles_bitexact(V.particles_to_host(out), p_o)
+        assert np.array_equal(counts.cpu().numpy(), c_o)
+        assert np.array_equal(nk.cpu().numpy(), nk_o)
+        assert np.array_equal(perm.cpu().numpy(), perm_o)
+
+
+def test_keyed_cycles_match_unkeyed(V):
+    """HotPath with the keyed sort (the default) and without: identical
+    particles after two sort periods (IEEE math)."""
+    from paper_conf_sc_tanlta25_b200.pic import HotPath
+    g = inputs.GridSpec(10, 8, 6, dt=0.5)
+    wl = inputs.Workload("keyed", g, [inputs.Species("electron", -1.0, 1.0, 0.5),
+                                      inputs.Species("ion", 1.0, 9.0, 0.1)], 20, 4, 4)
+    parts = inputs.make_species_particles(wl)
+    fields = inputs.make_fields(g, 0.05)
+    res = []
+    for keyed in (True, False):
+        hp = HotPath(wl, parts, fields, math=V.MATH_IEEE, keyed_sort=keyed)
+        hp.cycle(4)
+        hp.cycle(4)
+        torch.cuda.synchronize()
+        res.append([hp.particles_host(k) for k in range(2)])
+    for k in range(2):
+        assert_particles_bitexact(res[0][k], res[1][k])

@@ -599,3 +599,29 @@ def test_keyed_cycles_match_unkeyed(V):
         res.append([hp.particles_host(k) for k in range(2)])
     for k in range(2):
         assert_particles_bitexact(res[0][k], res[1][k])
+
+
+def test_advance_one_cta_per_sm_bitexact(V, orc):
+    """VPIC_OPT_ADVANCE_CTAS_PER_SM = 1 (half the persistent grid: every
+    warp takes twice the chunk pairs) gives the oracle's particles too."""
+    wl = inputs.config(0)
+    g = wl.grid
+    p = inputs.make_species_particles(wl)[0]
+    f = inputs.make_fields(g, 0.01)
+    interp_o = orc.load_interpolator(g, f.copy())
+    acc_o = np.zeros((g.nv, 12), np.float32)
+    acc_abs = np.zeros((g.nv, 12), np.float64)
+    p_o = p.copy()
+    orc.advance_p(g, -1.0, 1.0, p_o, interp_o, acc_o, acc_abs)
+    ctx = mkctx(V, g, V.MATH_IEEE, 2, 2)
+    ctx.set_option(V.VPIC_OPT_ADVANCE_CTAS_PER_SM, 1)
+    fd = torch.from_numpy(f.copy()).cuda()
+    interp = torch.zeros((g.nv, 24), dtype=torch.float32, device="cuda")
+    V.vpic_load_interpolator(ctx, fd, interp)
+    acc = torch.zeros((g.nv, 12), dtype=torch.float32, device="cuda")
+    pd = dev_particles(V, p)
+    nm = torch.zeros(1, dtype=torch.int64, device="cuda")
+    V.vpic_advance_p(ctx, -1.0, 1.0, pd, p.size, interp, acc, None, 0, nm, None)
+    torch.cuda.synchronize()
+    assert_particles_bitexact(V.particles_to_host(pd), p_o)
+    assert_acc_close(acc.cpu().numpy(), acc_o, acc_abs)

@@ -12,6 +12,18 @@
  * -O2 -ffp-contract=off (no FMA contraction), matching VPIC's FP32 arithmetic
  * (reading R16).  Where the oracle keeps checking quantities
  * (absolute-contribution sums, rho) it uses double.
+ *
+ * Pins (tests -m "not gpu"): every function below is pinned to
+ * something other than itself -- sort: hand-worked example + exhaustive
+ * brute force + the paper's run invariants; interpolator: closed forms;
+ * push: bit-exact uniform-E steps, TV2/TV3 golden values (tests/golden/),
+ * energy / gyration / E x B closed forms; move_p: geometry invariants and
+ * edge cases; deposit: the discrete continuity invariant and totals; unload
+ * and rho: single-slot / single-particle closed forms; remove_absorbed:
+ * numpy mask multiset; continuity residual: hand cases; field solver: Yee
+ * dispersion, div B, Gauss; gather-scatter: bincount / closed forms; the
+ * replay (orc_move_deposit) and all-core (orc_advance_p_omp) variants
+ * against the serial orc_advance_p.  No function is "parity unpinned".
  */
 #ifndef VPIC_ORACLE_H
 #define VPIC_ORACLE_H

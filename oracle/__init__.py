@@ -186,7 +186,7 @@ def move_deposit(spec, q, p, acc, acc_abs=None, max_movers=None):
     """The move + deposit half of advance_p on particles whose momenta are
     already pushed (in place on p and acc).  Returns movers."""
     assert p.dtype == PARTICLE_DTYPE and p.flags.c_contiguous
-    assert acc.dtype == np.float32 and acc.flags.c_contiguous
+    assert acc is None or (acc.dtype == np.float32 and acc.flags.c_contiguous)
     if max_movers is None:
         max_movers = p.size
     movers = np.zeros(max(max_movers, 1), MOVER_DTYPE)

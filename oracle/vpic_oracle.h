@@ -88,7 +88,8 @@ int64_t orc_advance_p_omp(const orc_grid *g, float q, float m, orc_particle *p, 
                           int nthreads);
 
 /* The move-and-deposit half of orc_advance_p alone: p[].u must already be
- * the pushed momentum (replay of another implementation's momenta). */
+ * the pushed momentum (replay of another implementation's momenta).  acc
+ * nullable: trajectories only (no deposit). */
 int64_t orc_move_deposit(const orc_grid *g, float qsp, orc_particle *p, int64_t np, float *acc,
                          double *acc_abs, double *acc_cond, orc_mover *movers,
                          int64_t max_movers);

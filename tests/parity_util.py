@@ -95,7 +95,7 @@ def replay_inputs(orc, g, q, p, p_gpu):
             if pat >> b & 1:
                 cand[comps[a]] = -cand[comps[a]]
         out = cand.copy()
-        orc.move_deposit(g, q, out, np.zeros((g.nv, 12), np.float32))
+        orc.move_deposit(g, q, out, None)          # trajectories only
         ok = (out.view(np.uint32).reshape(-1, 8) == p_gpu.view(np.uint32).reshape(-1, 8)).all(1)
         pick = ok & (chosen < 0)
         chosen[pick] = pat

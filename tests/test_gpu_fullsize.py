@@ -54,7 +54,7 @@ def test_fullsize_particles_sampled(orc, state):
         # T3: the bench arithmetic's move is the oracle's given the pushed
         # momenta -- every sampled particle's position and voxel bit for bit
         pr = replay_inputs(orc, g, sp.q, p0[idx].copy(), got)
-        orc.move_deposit(g, sp.q, pr, np.zeros((g.nv, 12), np.float32))
+        orc.move_deposit(g, sp.q, pr, None)
         assert_particles_bitexact(got, pr)
 
 

@@ -19,7 +19,8 @@ import pytest
 import torch
 
 from paper_conf_sc_tanlta25_b200 import inputs
-from parity_util import assert_acc_close, assert_particles_close, kick_bound, u_of
+from parity_util import (assert_acc_close, assert_particles_bitexact, assert_particles_close, kick_bound,
+                         replay_inputs, u_of)
 
 pytestmark = pytest.mark.gpu
 
@@ -60,6 +61,10 @@ def test_lpi_fullsize_particles_sampled(orc, lpi):
         acc = np.zeros((g.nv, 12), np.float32)
         orc.advance_p(g, sp.q, sp.m, ps, interp_o, acc)
         assert_particles_close(g, got, ps, u_of(p0[idx]), kick_bound(g, p0[idx], sp.q, sp.m, interp_o))
+        # T3: the move is the oracle's given the pushed momenta, bit for bit
+        pr = replay_inputs(orc, g, sp.q, p0[idx].copy(), got)
+        orc.move_deposit(g, sp.q, pr, None)
+        assert_particles_bitexact(got, pr)
 
 
 def test_lpi_fullsize_accumulator_sampled(orc, lpi):

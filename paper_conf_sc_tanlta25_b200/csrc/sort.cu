@@ -275,7 +275,14 @@ k_radix_pass(const KeyT *__restrict__ kin, const uint32_t *__restrict__ vin,
              KeyT *__restrict__ kout, uint32_t *__restrict__ vout, int64_t n, int shift,
              const uint32_t *__restrict__ dig_off, unsigned long long *__restrict__ status,
              unsigned int *__restrict__ tile_ctr, const int *__restrict__ live_bits) {
-  if (live_bits && shift > 0 && shift >= *live_bits) return;
+  if (live_bits) {
+    const int nb = *live_bits;
+    // the 32-bit and the 64-bit chain of rank passes are both launched; the
+    // key width the device found selects the one that runs
+    if (sizeof(KeyT) == 4 && nb > 32) return;
+    if (sizeof(KeyT) == 8 && nb <= 32) return;
+    if (shift > 0 && shift >= nb) return;
+  }
   constexpr int NB = 1 << BITS;
   extern __shared__ __align__(16) unsigned char smem[];
   uint16_t *whist = reinterpret_cast<uint16_t *>(smem);                       // [NW][NB]
@@ -451,12 +458,14 @@ __global__ void k_rank_setup(const uint32_t *__restrict__ K, int64_t n, int orde
 // Rank-pass keys (strided: r; tiled: (chunk - chunk0) * max_r + r) with the
 // digit histograms of the following (worst-case) passes; optional Alg. 1/2
 // new keys scattered to the INPUT index (perm_std[j]).
-template <class KeyT>
+// ckey: the rank keys as uint32 when they fit 32 bits (rp->nbits <= 32), as
+// uint64 otherwise (the buffer holds either).
 __global__ void __launch_bounds__(256)
 k_rank_keys(const uint32_t *__restrict__ K, const uint32_t *__restrict__ perm_std,
             const uint32_t *__restrict__ offs, int64_t n, int order, int64_t T,
-            const RankParams *__restrict__ rp, KeyT *__restrict__ ckey, PassDesc pd,
+            const RankParams *__restrict__ rp, void *__restrict__ ckey, PassDesc pd,
             uint32_t *__restrict__ ghist, int64_t *__restrict__ new_keys) {
+  using KeyT = uint64_t;
   extern __shared__ uint32_t sh[];
   int off[MAX_PASSES];
   int tot = 0;
@@ -467,6 +476,7 @@ k_rank_keys(const uint32_t *__restrict__ K, const uint32_t *__restrict__ perm_st
   const int64_t min_k = rp->min_k, max_k = rp->max_k, chunk0 = rp->chunk0;
   const uint64_t max_r = rp->max_r;
   const int nbits = rp->nbits;
+  const bool wide = nbits > 32;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t base = (int64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31); base < n;
        base += stride) {
@@ -483,7 +493,8 @@ k_rank_keys(const uint32_t *__restrict__ K, const uint32_t *__restrict__ perm_st
         ck = (KeyT)((uint64_t)(k / T - chunk0) * max_r + (uint64_t)r);
         if (new_keys) new_keys[perm_std[j]] = (k / T) * (T * (int64_t)max_r) + r * T + (k - min_k);
       }
-      ckey[j] = ck;
+      if (wide) static_cast<uint64_t *>(ckey)[j] = ck;
+      else static_cast<uint32_t *>(ckey)[j] = (uint32_t)ck;
     }
     for (int q = 0; q < pd.npass; ++q) {
       if (pd.shift[q] > 0 && pd.shift[q] >= nbits) break;   // skipped pass (uniform)
@@ -733,10 +744,12 @@ PassDesc rank_passes(int nbits) {
 
 // The rank stage of STRIDED / TILED_STRIDED: keys from the standard order
 // (K, P), passes sized on the device; returns the two candidate perm buffers
-// (the first when the number of live passes is even).
-template <class KeyT>
+// (the first when the number of live passes is even).  Rank keys go through
+// 32-bit passes when the device finds they fit (always for STRIDED), else
+// through 64-bit ones (TILED_STRIDED with (chunks) x max_r >= 2^32): both
+// chains are launched, the other one returns at once.
 cudaError_t rank_stage(vpic_ctx *c, int64_t np, int order, int64_t T, int worst_bits,
-                       const uint32_t *K, uint32_t *P, KeyT *ckA, KeyT *ckB, uint32_t *vfree,
+                       const uint32_t *K, uint32_t *P, void *ckA, void *ckB, uint32_t *vfree,
                        const uint32_t *offs, const unsigned int *max_r_dev, RankParams *rp,
                        uint32_t *ghist, uint32_t *goff, unsigned long long *status,
                        unsigned int *ctr, int64_t *new_keys, uint32_t **perm_even,
@@ -749,16 +762,22 @@ cudaError_t rank_stage(vpic_ctx *c, int64_t np, int order, int64_t T, int worst_
   for (int q = 0; q < pr.npass; ++q) tot += 1 << pr.bits[q];
   static std::atomic<uint64_t> configured{0};
   once_per_device(configured, [] {
-    cudaFuncSetAttribute(k_rank_keys<KeyT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaFuncSetAttribute(k_rank_keys, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          4 * MAX_PASSES * (1 << MAX_BITS));
   });
-  k_rank_keys<KeyT><<<grid_cap(np, 256, c->num_sms, 2), 256, 4 * (size_t)tot, s>>>(
+  k_rank_keys<<<grid_cap(np, 256, c->num_sms, 2), 256, 4 * (size_t)tot, s>>>(
       K, P, offs, np, order, T, rp, ckA, pr, ghist, new_keys); note_launch();
   CK(cudaGetLastError());
-  KeyT *kf = nullptr;
-  uint32_t *vf = nullptr;
-  CK(lsd_sort<KeyT>(pr, np, ckA, ckB, P, vfree, P, ghist, goff, status, ctr, false, &rp->nbits,
-                    &kf, &vf, s));
+  PassDesc p32 = pr;
+  p32.npass = std::min(pr.npass, 4);
+  uint32_t *k32 = nullptr, *vf = nullptr;
+  CK(lsd_sort<uint32_t>(p32, np, static_cast<uint32_t *>(ckA), static_cast<uint32_t *>(ckB), P, vfree, P,
+                        ghist, goff, status, ctr, false, &rp->nbits, &k32, &vf, s));
+  if (pr.npass > 4) {
+    uint64_t *k64 = nullptr;
+    CK(lsd_sort<uint64_t>(pr, np, static_cast<uint64_t *>(ckA), static_cast<uint64_t *>(ckB), P, vfree, P,
+                          ghist, goff, status, ctr, false, &rp->nbits, &k64, &vf, s));
+  }
   *perm_even = P;       // live passes: 2, 4, ...
   *perm_odd = vfree;    //              1, 3, ...
   return cudaSuccess;
@@ -845,17 +864,13 @@ cudaError_t launch_sort(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_
     uint32_t *ck = (K == kA) ? kB : kA;
     uint32_t *vfree = (P == vA) ? vB : vA;
     uint32_t *Pe = nullptr, *Po = nullptr;
-    if (order == VPIC_SORT_STRIDED) {
-      // r < max_r <= np < 2^32
-      CK(rank_stage<uint32_t>(c, np, order, T, bits_for((uint64_t)(np - 1)), K, P, ck, K, vfree,
-                              offs, misc, rp, ghist, goff, status, ctr, new_keys, &Pe, &Po, s));
-    } else {
-      // (chunk - chunk0) max_r + r <= ((nv - 1) / T) np + np - 1, in 64 bits
-      const uint64_t worst = (uint64_t)((nv - 1) / T) * (uint64_t)np + (uint64_t)(np - 1);
-      CK(rank_stage<uint64_t>(c, np, order, T, bits_for(worst), K, P,
-                              reinterpret_cast<uint64_t *>(ck), reinterpret_cast<uint64_t *>(K), vfree,
-                              offs, misc, rp, ghist, goff, status, ctr, new_keys, &Pe, &Po, s));
-    }
+    // strided: r < max_r <= np < 2^32; tiled: (chunk - chunk0) max_r + r <=
+    // ((nv - 1) / T) np + np - 1, up to 64 bits (8-B key buffers)
+    const uint64_t worst = order == VPIC_SORT_STRIDED
+                               ? (uint64_t)(np - 1)
+                               : (uint64_t)((nv - 1) / T) * (uint64_t)np + (uint64_t)(np - 1);
+    CK(rank_stage(c, np, order, T, bits_for(worst), K, P, ck, K, vfree, offs, misc, rp, ghist, goff,
+                  status, ctr, new_keys, &Pe, &Po, s));
     P = Pe;
     P_alt = Po;
     sel = rp;

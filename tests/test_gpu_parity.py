@@ -625,3 +625,30 @@ def test_advance_one_cta_per_sm_bitexact(V, orc):
     torch.cuda.synchronize()
     assert_particles_bitexact(V.particles_to_host(pd), p_o)
     assert_acc_close(acc.cpu().numpy(), acc_o, acc_abs)
+
+
+def test_sort_tiled_64bit_rank_keys(V, orc):
+    """TILED_STRIDED whose rank keys (chunk - chunk0) * max_r + r exceed 32
+    bits (T = 1 over a 2^18-voxel key range, 20000 particles in one voxel):
+    the 64-bit chain of rank passes runs; bit-exact against the oracle."""
+    g = inputs.GridSpec(64, 64, 64)
+    lo, hi, mid = g.voxel(1, 1, 1), g.voxel(64, 64, 64), g.voxel(30, 31, 32)
+    p = inputs.random_particles(g, 20003, 91, vox=[mid])
+    p["i"][:2] = lo
+    p["i"][-1] = hi
+    p = inputs.shuffle(p, 92)
+    assert (hi - lo) * 20000 > 2**32
+    ctx = mkctx(V, g)
+    n = p.size
+    p_in = dev_particles(V, p)
+    p_out = torch.empty_like(p_in)
+    ws = torch.empty(V.vpic_sort_workspace_bytes(ctx, n, 2), dtype=torch.uint8, device="cuda")
+    nk = torch.empty(n, dtype=torch.int64, device="cuda")
+    perm = torch.empty(n, dtype=torch.int64, device="cuda")
+    V.vpic_sort_particles(ctx, p_in, p_out, n, 2, 1, ws, None, nk, perm)
+    torch.cuda.synchronize()
+    p_o, _, nk_o, perm_o = orc.sort_particles(g, p, 2, 1)
+    assert nk_o.max() >= 2**32
+    assert_particles_bitexact(V.particles_to_host(p_out), p_o)
+    assert np.array_equal(nk.cpu().numpy(), nk_o)
+    assert np.array_equal(perm.cpu().numpy(), perm_o)

@@ -188,8 +188,8 @@ int vpic_sort_particles(vpic_ctx *ctx, const vpic_particle_t *p_in, vpic_particl
                         int32_t *voxel_counts, int64_t *new_keys, int64_t *perm,
                         void *stream);
 
-/* vpic_sort_particles with the voxel key of every input particle supplied
- * (keys[np] uint32 device, 4-B aligned -- e.g. written by the last
+/* vpic_sort_particles with the voxel key of every input
+ * particle supplied (keys[np] uint32 device, 4-B aligned -- e.g. written by the last
  * vpic_advance_p_keys of a sort period), so the sort does not read a 32-B
  * sector of every record to get its 4-B key (SURVEY.md §8(a) a1 fused into
  * the push).  keys[i] must equal p_in[i].i; otherwise identical to
@@ -231,8 +231,9 @@ int vpic_advance_p(vpic_ctx *ctx, float q, float m, vpic_particle_t *p, int64_t 
                    const float *interp, float *acc, vpic_mover_t *movers, int64_t max_movers,
                    int64_t *n_movers, int32_t *flags, void *stream);
 
-/* vpic_advance_p that also writes keys_out[i] = p[i].i as the call leaves
- * particle i (keys_out[np] uint32 device, 4-B aligned): the keys of the next
+/* vpic_advance_p that also writes keys_out[i] = p[i].i as the call
+ * leaves particle i (keys_out[np] uint32 device, 4-B aligned): the "copy of
+ * the keys" the next sort starts from, handed to
  * vpic_sort_particles_keyed, at the cost of a coalesced 4-B store per
  * particle.  Valid for that sort only if the call produced no movers (a
  * mover's record holds its stop code and vpic_migrate_particles reorders the

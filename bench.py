@@ -343,6 +343,7 @@ def our_arm(args, rank, world):
                  field_solve=args.field_solve, loopback_exchange=args.loopback and world == 1,
                  concurrent_species=args.concurrent_species,
                  device_exchange=args.exchange in ("auto", "device") and (world > 1 or args.loopback),
+                 device_exchange_fallback=args.exchange == "auto",
                  single_round=args.migration in ("auto", "single") and (world > 1 or args.loopback))
     hp.ctx.set_option(vpic.VPIC_OPT_ADVANCE_KERNEL, {"auto": 0, "direct": 1, "tma": 2}[args.kernel])
     n_local = hp.n_particles
@@ -488,7 +489,7 @@ def our_arm(args, rank, world):
                                    else f"domain{world}"),
                    "box_cells": [box.nx, box.ny, box.nz],
                    "field_solve": bool(args.field_solve),
-                   "exchange": ("nccl" if args.exchange == "nccl" else "device")
+                   "exchange": ("nccl" if (args.exchange == "nccl" or not hp.device_exchange) else "device")
                                if (world > 1 or args.loopback) else "none",
                    "migration": ("rounds" if args.migration == "rounds" else "single")
                                 if (world > 1 or args.loopback) else "none",

@@ -85,7 +85,7 @@ class HotPath:
                  device: Optional[int] = None, field_solve: bool = False, eps0: float = 1.0,
                  loopback_exchange: bool = False, concurrent_species: bool = False,
                  device_exchange: bool = False, inbox_cap: int = 0, single_round: bool = False,
-                 graphs: bool = False, keyed_sort: bool = True):
+                 graphs: bool = False, keyed_sort: bool = True, device_exchange_fallback: bool = False):
         vpic.load()
         self.wl = wl
         self.g = wl.grid
@@ -109,8 +109,20 @@ class HotPath:
             self.ctx.set_option(vpic.VPIC_OPT_LOOPBACK_EXCHANGE, 1)
         if single_round:        # moves finished in the ghost layer, one 26-neighbour exchange
             self.ctx.set_option(vpic.VPIC_OPT_SINGLE_ROUND_MIGRATION, 1)
+        self.exchange_note = None
         if device_exchange:     # movers stored into the neighbours' inboxes by the push (f4)
-            self.ctx.set_option(vpic.VPIC_OPT_DEVICE_EXCHANGE, inbox_cap if inbox_cap > 1 else 1)
+            try:
+                self.ctx.set_option(vpic.VPIC_OPT_DEVICE_EXCHANGE, inbox_cap if inbox_cap > 1 else 1)
+            except vpic.VpicError as e:
+                if not device_exchange_fallback:
+                    raise
+                # peers not load/store reachable (no NVLink / symmetric memory):
+                # the NCCL send/recv exchange of the same migration mode
+                device_exchange = False
+                self.exchange_note = f"device-initiated exchange unavailable ({e}); NCCL send/recv used"
+                import sys
+                print(f"HotPath: {self.exchange_note}", file=sys.stderr, flush=True)
+        self.device_exchange = device_exchange
         self.migrate = (nranks > 1 or loopback_exchange
                         or any(b == inputs.BC_ABSORB for b in self.g.pbc))
         # species pushed concurrently on their own streams, each persistent

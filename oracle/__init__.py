@@ -39,7 +39,11 @@ class OrcGrid(ctypes.Structure):
 
 def build(force: bool = False) -> str:
     """Compile liboracle.so (g++ -O2 -ffp-contract=off: no FMA contraction;
-    -fopenmp for the all-core baseline orc_advance_p_omp only)."""
+    -fopenmp for the all-core baseline orc_advance_p_omp only).
+    ORACLE_LIB (dev: tools/oracle_mutations.py) names a prebuilt library to
+    load instead -- a deliberately broken oracle the pins must reject."""
+    if os.environ.get("ORACLE_LIB"):
+        return os.environ["ORACLE_LIB"]
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < max(
             os.path.getmtime(_SRC), os.path.getmtime(os.path.join(_HERE, "vpic_oracle.h"))):
         cmd = ["g++", "-O2", "-std=c++17", "-ffp-contract=off", "-fno-fast-math", "-fopenmp",

@@ -420,3 +420,143 @@ def test_advance_p_omp_matches_serial(orc, threads):
     assert np.all(np.abs(a1.astype(np.float64) - a2) <= 1e-5 * aa + 1e-30)
     assert np.array_equal(np.sort(m1.view(np.uint32).reshape(-1, 4), axis=0),
                           np.sort(m2.view(np.uint32).reshape(-1, 4), axis=0)) and m1.size > 0
+
+
+# ------------------------------------------------ gather / geometry pins --
+def _edge_field_push(orc, comp, coef, g, p):
+    """One step from rest with E only (B = 0): u = 2 qdt_2mc E(particle)."""
+    f = np.zeros((g.nv, 8), np.float32)
+    z, y, x = np.meshgrid(np.arange(g.nz + 2), np.arange(g.ny + 2), np.arange(g.nx + 2), indexing="ij")
+    X = {"x": x, "y": y, "z": z}
+    a, b, c, d, t1, t2 = coef
+    f[:, comp] = (a + b * X[t1] + c * X[t2] + d * X[t1] * X[t2]).reshape(-1).astype(np.float32)
+    interp = orc.load_interpolator(g, f)
+    acc = np.zeros((g.nv, 12), np.float32)
+    q = p.copy()
+    orc.advance_p(g, 1.0, 1.0, q, interp, acc)
+    return q
+
+
+@pytest.mark.parametrize("comp,t1,t2", [(0, "y", "z"), (1, "z", "x"), (2, "x", "y")])
+def test_gather_bilinear_E_closed_form(orc, comp, t1, t2):
+    """The gather ("gather phase"): E_a on the a-edges of a voxel,
+    bilinear in the two transverse coordinates, is interpolated exactly at
+    the particle -- E_a(particle) = f(x_t1 + (1+d_t1)/2, x_t2 + (1+d_t2)/2) for
+    edge values f(X_t1, X_t2) = a + b X_t1 + c X_t2 + d X_t1 X_t2 (edge a of
+    voxel (x,y,z) sits at node coordinates (x_t1, x_t2) transversely).  One
+    step from rest with B = 0 gives u_a = 2 qdt_2mc E_a exactly (to float)."""
+    # walls (the caller owns their ghost planes: the field stays bilinear up
+    # to the last edge), particles away from them (no reflection in a step)
+    g = inputs.GridSpec(6, 5, 7, dt=0.5, pbc=(1,) * 6)   # non-cubic counts: no axis symmetry
+    inner = [g.voxel(x, y, z) for z in range(2, 7) for y in range(2, 5) for x in range(2, 6)]
+    p = inputs.random_particles(g, 400, 11, vox=inner)
+    p["ux"] = p["uy"] = p["uz"] = 0
+    coef = (0.01, 0.003, -0.002, 0.0007, t1, t2)
+    q = _edge_field_push(orc, comp, coef, g, p)
+    xyz = dict(zip("xyz", g.coords(p["i"])))
+    off = {"x": p["dx"].astype(np.float64), "y": p["dy"].astype(np.float64), "z": p["dz"].astype(np.float64)}
+    X1 = xyz[t1] + (1 + off[t1]) / 2
+    X2 = xyz[t2] + (1 + off[t2]) / 2
+    E = coef[0] + coef[1] * X1 + coef[2] * X2 + coef[3] * X1 * X2
+    qdt_2mc = 0.5 / 2
+    names = ("ux", "uy", "uz")
+    assert np.abs(q[names[comp]] - 2 * qdt_2mc * E).max() < 3e-8
+    for k in range(3):
+        if k != comp:
+            assert np.all(q[names[k]] == 0)
+
+
+@pytest.mark.parametrize("axis", [0, 1, 2])
+def test_gather_linear_B_closed_form(orc, axis):
+    """cB_a is linear along its face normal inside the voxel: at the particle
+    cB_a = cb(x_a + (1+d_a)/2) for face values cb(X_a) = a + b X_a.  A
+    particle moving perpendicular to B rotates by theta = 2 atan(v3 |cB|)
+    per step (pinned by TV2) -- checked against the closed-form |cB| at its
+    position."""
+    g = inputs.GridSpec(6, 5, 7, dt=0.5, pbc=(1,) * 6)
+    inner = [g.voxel(x, y, z) for z in range(2, 7) for y in range(2, 5) for x in range(2, 6)]
+    p = inputs.random_particles(g, 200, 12, vox=inner)
+    names = ("ux", "uy", "uz")
+    for k in range(3):
+        p[names[k]] = 0
+    perp = (axis + 1) % 3
+    p[names[perp]] = 0.2
+    f = np.zeros((g.nv, 8), np.float32)
+    z, y, x = np.meshgrid(np.arange(g.nz + 2), np.arange(g.ny + 2), np.arange(g.nx + 2), indexing="ij")
+    X = (x, y, z)[axis]
+    f[:, 4 + axis] = (0.5 + 0.1 * X).reshape(-1).astype(np.float32)
+    interp = orc.load_interpolator(g, f)
+    acc = np.zeros((g.nv, 12), np.float32)
+    q = p.copy()
+    orc.advance_p(g, 1.0, 1.0, q, interp, acc)
+    Xa = g.coords(p["i"])[axis] + (1 + p[("dx", "dy", "dz")[axis]].astype(np.float64)) / 2
+    B = 0.5 + 0.1 * Xa
+    qdt_2mc = 0.25
+    gam = np.sqrt(1 + 0.04)
+    v0 = qdt_2mc / gam
+    v2 = v0 * v0 * B * B
+    v3 = v0 * (1 + v2 * (1 / 3 + v2 * 2 / 15))
+    theta = 2 * np.arctan(v3 * B)
+    other = (axis + 2) % 3
+    got = np.arctan2(np.abs(q[names[other]].astype(np.float64)), q[names[perp]].astype(np.float64))
+    assert np.abs(got - theta).max() < 1e-5
+
+
+def test_half_displacement_per_axis_on_noncubic_cells(orc):
+    """The position advance uses c dt / d_a on each axis (VPIC's cdt_dx,
+    cdt_dy, cdt_dz): on cells of 0.5 x 1 x 2 a particle at constant velocity
+    moves u_a c dt / gamma physical units along each axis per step."""
+    g = inputs.GridSpec(6, 5, 4, dx=0.5, dy=1.0, dz=2.0, dt=0.2)
+    p = np.zeros(1, PD)
+    p["i"] = g.voxel(3, 3, 2)
+    p["ux"], p["uy"], p["uz"] = 0.3, -0.2, 0.25
+    p["w"] = 1
+    x0 = np.array([(p["dx"][0] + 1) / 2 * 0.5, (p["dy"][0] + 1) / 2 * 1.0, (p["dz"][0] + 1) / 2 * 2.0])
+    interp = orc.load_interpolator(g, np.zeros((g.nv, 8), np.float32))
+    acc = np.zeros((g.nv, 12), np.float32)
+    q = p.copy()
+    orc.advance_p(g, 1.0, 1.0, q, interp, acc)
+    assert q["i"][0] == p["i"][0]
+    x1 = np.array([(q["dx"][0] + 1) / 2 * 0.5, (q["dy"][0] + 1) / 2 * 1.0, (q["dz"][0] + 1) / 2 * 2.0])
+    u = np.array([0.3, -0.2, 0.25])
+    assert np.abs((x1 - x0) - u * 0.2 / np.sqrt(1 + u @ u)).max() < 1e-7
+
+
+def test_track_ending_exactly_on_a_face_stays(orc):
+    """Reading R13: a track whose end lands exactly on a face (d + 2 disp ==
+    1 in float) is not a crossing -- the end of track wins the tie with 2:
+    the particle stays in its voxel with the offset exactly +1."""
+    g = grid(n=4, dt=0.5)
+    f32 = np.float32
+    disp = (f32(1.0) * f32(0.5)) * (f32(1.0) / np.sqrt(f32(1.0) + f32(1.0) * f32(1.0)))
+    d = f32(1.0) - f32(2.0) * disp
+    for _ in range(8):
+        e = (d + disp) + disp
+        if e == f32(1.0):
+            break
+        d = np.nextafter(d, f32(2.0) if e < 1 else f32(-2.0), dtype=np.float32)
+    p = one_particle(g, d=(float(d), 0.0, 0.0), u=(1.0, 0.0, 0.0))
+    interp = orc.load_interpolator(g, uniform_fields(g))
+    acc = np.zeros((g.nv, 12), np.float32)
+    v0 = p["i"][0]
+    orc.advance_p(g, 1.0, 1.0, p, interp, acc)
+    assert p["i"][0] == v0 and p["dx"][0] == np.float32(1.0)
+
+
+def test_move_p_end_of_track_ties_with_two(orc):
+    """Reading R13 inside move_p: a streak whose end lies exactly on a face
+    (fraction to the face == 2, the end-of-track value) ends the move -- the
+    particle stays in its voxel on the face, it does not cross (d = 0.5,
+    remaining half-displacement 0.25: (1 - 0.5) / 0.25 = 2 exactly)."""
+    g = grid(n=4, dt=0.5)
+    acc = np.zeros((g.nv, 12), np.float32)
+    for axis in range(3):
+        d = [0.0, 0.0, 0.0]
+        r = [0.0, 0.0, 0.0]
+        d[axis], r[axis] = 0.5, 0.25
+        p = one_particle(g, d=tuple(d))
+        v0 = p["i"][0]
+        mv = _mover(tuple(r))
+        assert orc.move_p(g, p, mv, acc, 1.0) == 0
+        assert p["i"][0] == v0
+        assert (p["dx"][0], p["dy"][0], p["dz"][0])[axis] == np.float32(1.0)

@@ -152,6 +152,12 @@ def adv_cases():
     wp, pp = lpi_small()
     out.append(("lpi_slab_electrons", wp.grid, pp[0], -1.0, 1.0,
                 inputs.make_fields(wp.grid, 0.01, kind="lpi")))
+    # non-cubic cells (every cdt/d and cell-size factor distinct; dt under the
+    # Courant limit of the smallest cell)
+    R = inputs.BC_REFLECT
+    gn = inputs.GridSpec(8, 7, 6, dx=0.6, dy=1.4, dz=1.0, dt=0.4, pbc=(0, R, 0, 0, R, 0))
+    out.append(("noncubic_cells", gn, inputs.random_particles(gn, 15000, 14, u_scale=0.8), -1.0, 1.0,
+                inputs.make_fields(gn, 0.05, seed=6)))
     # random order on 40^3 voxels: every warp's items in distinct voxels
     gs = inputs.GridSpec(40, 40, 40)
     out.append(("scattered_cache_overflow", gs, inputs.random_particles(gs, 150000, 13, u_scale=0.5),

@@ -162,6 +162,19 @@ def adv_cases():
     gs = inputs.GridSpec(40, 40, 40)
     out.append(("scattered_cache_overflow", gs, inputs.random_particles(gs, 150000, 13, u_scale=0.5),
                 -1.0, 1.0, inputs.make_fields(gs, 0.02, seed=5)))
+    # voxel-sorted, ~125 per voxel, with items moved into the x-neighbour voxel
+    # where they sit (crossed since the sort): 5% in the first half (chunks of
+    # the carry-first deposit, <= 24 stragglers), 40% in the second (chunks of
+    # the general segment loop), voxels changing inside chunks
+    gq = inputs.GridSpec(8, 8, 8)
+    pq = inputs.random_particles(gq, 64000, 15, u_scale=0.3)
+    pq = pq[np.argsort(pq["i"], kind="stable")]
+    rng = np.random.default_rng(16)
+    frac = np.where(np.arange(pq.size) < pq.size // 2, 0.05, 0.40)
+    mv = rng.random(pq.size) < frac
+    x = pq["i"] % (gq.nx + 2)
+    pq["i"] = np.where(mv, pq["i"] + np.where(x < gq.nx, 1, -1), pq["i"])
+    out.append(("sorted_stragglers", gq, pq, -1.0, 1.0, inputs.make_fields(gq, 0.02, seed=7)))
     return out
 
 

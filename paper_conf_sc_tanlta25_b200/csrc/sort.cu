@@ -269,12 +269,28 @@ __global__ void k_scan_hist(const uint32_t *__restrict__ ghist, uint32_t *__rest
 // live_bits (nullable): the pass returns at once (every CTA) when its digit
 // lies above the key width the device found (*live_bits), so the host can
 // launch the worst-case number of passes without reading it back.
-template <int BITS, class KeyT>
+// REC (the last pass of the standard order): instead of the permutation,
+// the pass moves the 32-B records themselves -- out[pos] = in[val] -- in its
+// coalesced digit-run scatter (two lanes per record, RILP half-records in
+// flight per thread), plus the optional int64 permutation: the record gather
+// is fused into the pass (no permutation written and re-read, one launch
+// less, the gather's DRAM-bound random reads overlap the ranking).
+struct RecMove {
+  const vpic_particle_t *in;
+  vpic_particle_t *out;
+  int64_t *perm64;
+};
+#ifndef VPIC_SORT_RILP
+#define VPIC_SORT_RILP 4
+#endif
+constexpr int RILP = VPIC_SORT_RILP;
+
+template <int BITS, class KeyT, bool REC = false>
 __global__ void __launch_bounds__(NT, VPIC_SORT_MINB)
 k_radix_pass(const KeyT *__restrict__ kin, const uint32_t *__restrict__ vin,
              KeyT *__restrict__ kout, uint32_t *__restrict__ vout, int64_t n, int shift,
              const uint32_t *__restrict__ dig_off, unsigned long long *__restrict__ status,
-             unsigned int *__restrict__ tile_ctr, const int *__restrict__ live_bits) {
+             unsigned int *__restrict__ tile_ctr, const int *__restrict__ live_bits, RecMove rec) {
   if (live_bits) {
     const int nb = *live_bits;
     // the 32-bit and the 64-bit chain of rank passes are both launched; the
@@ -409,12 +425,50 @@ k_radix_pass(const KeyT *__restrict__ kin, const uint32_t *__restrict__ vin,
     __syncthreads();
     const int64_t t0 = tile * TILE;
     const int nvalid = (int)(n - t0 < TILE ? n - t0 : (int64_t)TILE);
-    for (int e = threadIdx.x; e < nvalid; e += NT) {
-      const KeyT k = skey[e];
-      const uint32_t d = (uint32_t)((k >> shift) & (NB - 1));
-      const uint32_t pos = tpref[d] + (uint32_t)e - tstart[d];
-      if (kout) kout[pos] = k;
-      vout[pos] = sval[e];
+    if (REC) {
+      // half-record h of element e: lanes 2j, 2j+1 move one whole record
+      const float4 *src = reinterpret_cast<const float4 *>(rec.in);
+      float4 *dst = reinterpret_cast<float4 *>(rec.out);
+      for (int tb = 0; tb < 2 * nvalid; tb += NT * RILP) {
+        uint32_t sidx[RILP], dpos[RILP];
+        float4 v[RILP];
+#pragma unroll
+        for (int j = 0; j < RILP; ++j) {
+          const int t = tb + j * NT + (int)threadIdx.x;
+          if (t < 2 * nvalid) {
+            const int e = t >> 1;
+            const KeyT k = skey[e];
+            const uint32_t d = (uint32_t)((k >> shift) & (NB - 1));
+            dpos[j] = tpref[d] + (uint32_t)e - tstart[d];
+            sidx[j] = sval[e];
+          }
+        }
+#pragma unroll
+        for (int j = 0; j < RILP; ++j) {
+          const int t = tb + j * NT + (int)threadIdx.x;
+          if (t < 2 * nvalid) {
+            const float4 *a = src + 2 * (int64_t)sidx[j] + (t & 1);
+            asm volatile("ld.global.nc.L2::64B.v4.f32 {%0,%1,%2,%3}, [%4];"
+                         : "=f"(v[j].x), "=f"(v[j].y), "=f"(v[j].z), "=f"(v[j].w) : "l"(a));
+          }
+        }
+#pragma unroll
+        for (int j = 0; j < RILP; ++j) {
+          const int t = tb + j * NT + (int)threadIdx.x;
+          if (t < 2 * nvalid) {
+            __stcs(dst + 2 * (int64_t)dpos[j] + (t & 1), v[j]);
+            if (rec.perm64 && !(t & 1)) rec.perm64[dpos[j]] = sidx[j];
+          }
+        }
+      }
+    } else {
+      for (int e = threadIdx.x; e < nvalid; e += NT) {
+        const KeyT k = skey[e];
+        const uint32_t d = (uint32_t)((k >> shift) & (NB - 1));
+        const uint32_t pos = tpref[d] + (uint32_t)e - tstart[d];
+        if (kout) kout[pos] = k;
+        vout[pos] = sval[e];
+      }
     }
 #if VPIC_SORT_PERSIST
     if (next >= ntiles) break;
@@ -650,16 +704,16 @@ PassDesc make_passes(int nbits) {
   return pd;
 }
 
-template <int BITS, class KeyT>
+template <int BITS, class KeyT, bool REC>
 cudaError_t radix_pass_bits(const KeyT *kin, const uint32_t *vin, KeyT *kout, uint32_t *vout,
                             int64_t n, int shift, const uint32_t *dig_off,
                             unsigned long long *status, unsigned int *ctr, const int *live_bits,
-                            cudaStream_t s) {
+                            cudaStream_t s, RecMove rec) {
   const size_t smem = (size_t)NW * (1 << BITS) * 2 + (size_t)(1 << BITS) * 8 + (size_t)TILE * (sizeof(KeyT) + 4);
   const int64_t tiles = (n + TILE - 1) / TILE;
   static std::atomic<uint64_t> configured{0};   // > 48 KB only for large tiles; once per device
   once_per_device(configured, [&] {
-    cudaFuncSetAttribute(k_radix_pass<BITS, KeyT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(k_radix_pass<BITS, KeyT, REC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   });
   int64_t grid = tiles;
 #if VPIC_SORT_PERSIST
@@ -667,21 +721,23 @@ cudaError_t radix_pass_bits(const KeyT *kin, const uint32_t *vin, KeyT *kout, ui
     int dev = 0, sms = 0, per_sm = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_radix_pass<BITS, KeyT>, NT, smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_radix_pass<BITS, KeyT, REC>, NT, smem);
     grid = std::min<int64_t>(tiles, (int64_t)sms * std::max(per_sm, 1));
   }
 #endif
-  k_radix_pass<BITS, KeyT><<<(unsigned)grid, NT, smem, s>>>(kin, vin, kout, vout, n, shift, dig_off,
-                                                             status, ctr, live_bits); note_launch();
+  k_radix_pass<BITS, KeyT, REC><<<(unsigned)grid, NT, smem, s>>>(kin, vin, kout, vout, n, shift, dig_off,
+                                                                  status, ctr, live_bits, rec); note_launch();
   return cudaGetLastError();
 }
 
 template <class KeyT>
 cudaError_t radix_pass(int bits, const KeyT *kin, const uint32_t *vin, KeyT *kout, uint32_t *vout,
                        int64_t n, int shift, const uint32_t *dig_off, unsigned long long *status,
-                       unsigned int *ctr, const int *live_bits, cudaStream_t s) {
+                       unsigned int *ctr, const int *live_bits, cudaStream_t s, const RecMove *rec = nullptr) {
+  const RecMove r0{nullptr, nullptr, nullptr};
   switch (bits) {
-#define VPIC_RP(B) case B: return radix_pass_bits<B, KeyT>(kin, vin, kout, vout, n, shift, dig_off, status, ctr, live_bits, s);
+#define VPIC_RP(B) case B: return rec ? radix_pass_bits<B, KeyT, true>(kin, vin, kout, vout, n, shift, dig_off, status, ctr, live_bits, s, *rec) \
+                                      : radix_pass_bits<B, KeyT, false>(kin, vin, kout, vout, n, shift, dig_off, status, ctr, live_bits, s, r0);
     VPIC_RP(1) VPIC_RP(2) VPIC_RP(3) VPIC_RP(4) VPIC_RP(5) VPIC_RP(6) VPIC_RP(7) VPIC_RP(8)
 #undef VPIC_RP
     default: return cudaErrorInvalidValue;
@@ -708,7 +764,8 @@ cudaError_t lsd_sort(const PassDesc &pd, int64_t n, KeyT *kA, KeyT *kB, uint32_t
                      uint32_t *vB, const uint32_t *vals0, uint32_t *ghist, uint32_t *goff,
                      unsigned long long *status, unsigned int *ctr, bool need_keys_out,
                      const int *live_bits, KeyT **k_final, uint32_t **v_final, cudaStream_t s,
-                     const KeyT *k_first = nullptr /* the first pass's keys, if not in kA */) {
+                     const KeyT *k_first = nullptr /* the first pass's keys, if not in kA */,
+                     const RecMove *rec = nullptr /* the last pass moves the records */) {
   CK(cudaMemsetAsync(ctr, 0, 4 * MAX_PASSES, s));
   k_scan_hist<<<pd.npass, 256, 0, s>>>(ghist, goff, pd); note_launch();
   CK(cudaGetLastError());
@@ -721,7 +778,8 @@ cudaError_t lsd_sort(const PassDesc &pd, int64_t n, KeyT *kA, KeyT *kB, uint32_t
     CK(cudaMemsetAsync(status, 0, 8 * (size_t)tiles * (1 << pd.bits[q]), s));
     const bool last = q == pd.npass - 1;
     CK(radix_pass<KeyT>(pd.bits[q], q == 0 ? kin0 : kin, vin, (last && !need_keys_out) ? nullptr : kout,
-                        vout, n, pd.shift[q], goff + q * (1 << MAX_BITS), status, ctr + q, live_bits, s));
+                        vout, n, pd.shift[q], goff + q * (1 << MAX_BITS), status, ctr + q, live_bits, s,
+                        last ? rec : nullptr));
     *k_final = kout;
     *v_final = vout;
     std::swap(kin, kout);
@@ -846,8 +904,11 @@ cudaError_t launch_sort(vpic_ctx *c, const vpic_particle_t *p_in, vpic_particle_
   // ---- standard order: stable LSD radix sort of (voxel, index)
   uint32_t *K = nullptr, *P = nullptr;
   const bool need_offs = order != VPIC_SORT_STANDARD;
+  // standard order: the last pass moves the records (no separate gather)
+  const RecMove rec{p_in, p_out, perm};
   CK(lsd_sort<uint32_t>(pd, np, kA, kB, vA, vB, nullptr, ghist, goff, status, ctr, need_offs,
-                        nullptr, &K, &P, s, keys_in));
+                        nullptr, &K, &P, s, keys_in, need_offs ? nullptr : &rec));
+  if (!need_offs) return cudaSuccess;
   const RankParams *sel = nullptr;
   uint32_t *P_alt = nullptr;
   if (need_offs) {  // offs[k] = first standard position of voxel k; max_r

@@ -598,6 +598,18 @@ def test_keyed_sort_matches_sort(V, orc, order):
         assert np.array_equal(counts.cpu().numpy(), c_o)
         assert np.array_equal(nk.cpu().numpy(), nk_o)
         assert np.array_equal(perm.cpu().numpy(), perm_o)
+        if order == 0:
+            # no voxel histogram asked for: digit histograms straight from the keys
+            out2 = torch.empty_like(pd)
+            perm2 = torch.full((p.size,), -3, dtype=torch.int64, device="cuda")
+            V.vpic_sort_particles_keyed(ctx, pd, out2, p.size, order, T, keys, ws, None, None, perm2)
+            torch.cuda.synchronize()
+            assert_particles_bitexact(V.particles_to_host(out2), p_o)
+            assert np.array_equal(perm2.cpu().numpy(), perm_o)
+            out3 = torch.empty_like(pd)
+            V.vpic_sort_particles_keyed(ctx, pd, out3, p.size, order, T, keys, ws, None, None, None)
+            torch.cuda.synchronize()
+            assert_particles_bitexact(V.particles_to_host(out3), p_o)
 
 
 def test_keyed_cycles_match_unkeyed(V):

@@ -632,9 +632,40 @@ def test_keyed_cycles_match_unkeyed(V):
         assert_particles_bitexact(res[0][k], res[1][k])
 
 
+@pytest.mark.parametrize("deposit", [2, 3], ids=["warp", "smem"])
+def test_advance_runs_wrap_bitexact(V, orc, deposit):
+    """More chunk runs than warps (1 CTA per SM, 1.6 M voxel-sorted particles:
+    > 16 x 8 x 148 chunks), so every warp goes on to later runs (runs of 16
+    consecutive chunks in WARP mode, pairs in SMEM mode) and carries its
+    voxel across chunks: IEEE particles bit-exact, accumulator within T1."""
+    g = inputs.GridSpec(32, 32, 32)
+    p = inputs.random_particles(g, 1600000, 91, u_scale=0.3)
+    p = p[np.argsort(p["i"], kind="stable")]
+    f = inputs.make_fields(g, 0.02, seed=8)
+    interp_o = orc.load_interpolator(g, f.copy())
+    acc_o = np.zeros((g.nv, 12), np.float32)
+    acc_abs = np.zeros((g.nv, 12), np.float64)
+    p_o = p.copy()
+    orc.advance_p(g, -1.0, 1.0, p_o, interp_o, acc_o, acc_abs)
+    ctx = mkctx(V, g, V.MATH_IEEE, deposit, 2)
+    ctx.set_option(V.VPIC_OPT_ADVANCE_CTAS_PER_SM, 1)
+    assert 64 * 16 * 8 * ctx.info()["num_sms"] < p.size
+    fd = torch.from_numpy(f.copy()).cuda()
+    interp = torch.zeros((g.nv, 24), dtype=torch.float32, device="cuda")
+    V.vpic_load_interpolator(ctx, fd, interp)
+    acc = torch.zeros((g.nv, 12), dtype=torch.float32, device="cuda")
+    pd = dev_particles(V, p)
+    nm = torch.zeros(1, dtype=torch.int64, device="cuda")
+    V.vpic_advance_p(ctx, -1.0, 1.0, pd, p.size, interp, acc, None, 0, nm, None)
+    torch.cuda.synchronize()
+    assert int(nm.item()) == 0
+    assert_particles_bitexact(V.particles_to_host(pd), p_o)
+    assert_acc_close(acc.cpu().numpy(), acc_o, acc_abs)
+
+
 def test_advance_one_cta_per_sm_bitexact(V, orc):
-    """VPIC_OPT_ADVANCE_CTAS_PER_SM = 1 (half the persistent grid: every
-    warp takes twice the chunk pairs) gives the oracle's particles too."""
+    """VPIC_OPT_ADVANCE_CTAS_PER_SM = 1 (half the persistent grid) gives the
+    oracle's particles too."""
     wl = inputs.config(0)
     g = wl.grid
     p = inputs.make_species_particles(wl)[0]

@@ -49,6 +49,16 @@ MUTATIONS = [
     ("smem deposit: segment sum to the neighbouring slot", "advance_p.cu",
      "      if (!(lane & 1) && lane < 24) red_add(acc + 12 * (int64_t)seg + (lane >> 1), sum);\n    }\n    doneA",
      "      if (!(lane & 1) && lane < 24) red_add(acc + 12 * (int64_t)seg + ((lane >> 1) ^ 1), sum);\n    }\n    doneA"),
+    ("carry-first: stragglers of set A not deposited", "advance_p.cu",
+     "        if (sA) deposit_lane(acc, keyA, cA);", "        (void)sA;"),
+    ("carry-first: A items of the carried voxel dropped", "advance_p.cu",
+     "        if (inCA) t += cA[j];", "        (void)inCA;"),
+    ("carry-first: B items of the chunk's last voxel not carried", "advance_p.cu",
+     "          if (inLB) t += cB[j];", "          (void)inLB;"),
+    ("carry-first: new carry keeps the old voxel", "advance_p.cu",
+     "        cr->key = last;", "        cr->key = ck >= 0 ? ck : last;"),
+    ("chunk runs: the next run starts one chunk late", "advance_p.cu",
+     "c + RUN * GW - (RUN - 1)", "c + RUN * GW - (RUN - 2)"),
     ("TMA kernel: B crossers queued over A's slots", "advance_p.cu",
      "wrapn<QCAP>(qhead + qn + __popc(cmA) + __popc(cmB & lt))", "wrapn<QCAP>(qhead + qn + __popc(cmB & lt))"),
     ("TMA kernel: B keys written to A's slots", "advance_p.cu",
@@ -80,9 +90,14 @@ MUTATIONS = [
     # ---- sort (sort.cu)
     ("radix rank counts later lanes (unstable)", "sort.cu",
      "      const uint32_t r = cur + __popc(peers & lt);", "      const uint32_t r = cur + __popc(peers & ~lt & ~(1u << lane));"),
-    ("gather swaps the record halves", "sort.cu",
-     "        const float4 *a = src + 2 * (int64_t)sidx[j] + (t & 1);",
-     "        const float4 *a = src + 2 * (int64_t)sidx[j] + ((t & 1) ^ 1);"),
+    ("gather (strided / tiled orders) swaps the record halves", "sort.cu",
+     "\n        const float4 *a = src + 2 * (int64_t)sidx[j] + (t & 1);",
+     "\n        const float4 *a = src + 2 * (int64_t)sidx[j] + ((t & 1) ^ 1);"),
+    ("fused record pass (standard order) swaps the record halves", "sort.cu",
+     "\n            const float4 *a = src + 2 * (int64_t)sidx[j] + (t & 1);",
+     "\n            const float4 *a = src + 2 * (int64_t)sidx[j] + ((t & 1) ^ 1);"),
+    ("fused record pass: permutation written one slot off", "sort.cu",
+     "rec.perm64[dpos[j]] = sidx[j];", "rec.perm64[dpos[j] ^ 1] = sidx[j];"),
     ("tiled rank key: chunk from key - min_k (R4)", "sort.cu",
      "        ck = (KeyT)((uint64_t)(k / T - chunk0) * max_r + (uint64_t)r);",
      "        ck = (KeyT)((uint64_t)((k - min_k) / T) * max_r + (uint64_t)r);"),
@@ -93,17 +108,19 @@ UNITS = {"advance_p.cu": ["advance_fast.o", "advance_ieee.o"], "exact_math.cuh":
          "diagnostics.cu": ["diagnostics.o"]}
 
 TESTS = ("ieee_bitexact or fast_tolerance or sort_parity or edge_cases or unload_parity or ghost_fill "
-         "or keyed or sort_captures or chunk_edges or one_cta or 64bit or absorb_movers "
+         "or keyed or sort_captures or chunk_edges or one_cta or runs_wrap or 64bit or absorb_movers "
          "or test_gpu_fields or test_gpu_diagnostics")
 
 
-def build():
+def build(only=None):
     from paper_conf_sc_tanlta25_b200 import _build
     _build.build()
     inc, libdir = _build.nccl_dirs()
     units, I = _build._units()
     unit_flags = {o: (src, extra) for o, src, extra in units}
     for k, (name, fname, old, new) in enumerate(MUTATIONS):
+        if only is not None and k not in only:
+            continue
         path = os.path.join(PKG, "csrc", fname)
         src = open(path).read()
         if src.count(old) != 1:
@@ -133,11 +150,13 @@ def build():
         print(f"built mut{k}: {name}", flush=True)
 
 
-def run(out):
+def run(out, only=None):
     lines = []
     killed = total = 0
     todo = [(-1, ("control: the product library", None, None, None))] + list(enumerate(MUTATIONS))
     for k, (name, fname, old, new) in todo:
+        if only is not None and k >= 0 and k not in only:
+            continue
         lib = os.path.join(PKG, "libvpic.so" if k < 0 else f"libvpic_mut{k}.so")
         if not os.path.exists(lib):
             continue
@@ -177,5 +196,6 @@ if __name__ == "__main__":
     ap = argparse.ArgumentParser()
     ap.add_argument("cmd", choices=["build", "run"])
     ap.add_argument("--out", default=None)
+    ap.add_argument("--only", type=int, nargs="*", default=None, help="mutation indices")
     a = ap.parse_args()
-    build() if a.cmd == "build" else run(a.out)
+    build(a.only) if a.cmd == "build" else run(a.out, a.only)

@@ -441,6 +441,7 @@ k_radix_pass(const KeyT *__restrict__ kin, const uint32_t *__restrict__ vin,
             const uint32_t d = (uint32_t)((k >> shift) & (NB - 1));
             dpos[j] = tpref[d] + (uint32_t)e - tstart[d];
             sidx[j] = sval[e];
+            VPIC_ASSERT((int64_t)dpos[j] < n && (int64_t)sidx[j] < n);
           }
         }
 #pragma unroll
@@ -466,6 +467,7 @@ k_radix_pass(const KeyT *__restrict__ kin, const uint32_t *__restrict__ vin,
         const KeyT k = skey[e];
         const uint32_t d = (uint32_t)((k >> shift) & (NB - 1));
         const uint32_t pos = tpref[d] + (uint32_t)e - tstart[d];
+        VPIC_ASSERT((int64_t)pos < n);
         if (kout) kout[pos] = k;
         vout[pos] = sval[e];
       }
@@ -612,6 +614,7 @@ k_gather(const vpic_particle_t *__restrict__ pin, vpic_particle_t *__restrict__ 
       // 64-B L2 fetch granularity: the neighbouring records of a source line
       // go to other output voxels, rarely still cached (-1% vs default/256 B)
       if (t < nh) {
+        VPIC_ASSERT((int64_t)sidx[j] < n);
         const float4 *a = src + 2 * (int64_t)sidx[j] + (t & 1);
         asm volatile("ld.global.nc.L2::64B.v4.f32 {%0,%1,%2,%3}, [%4];"
                      : "=f"(v[j].x), "=f"(v[j].y), "=f"(v[j].z), "=f"(v[j].w) : "l"(a));

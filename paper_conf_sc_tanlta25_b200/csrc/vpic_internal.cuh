@@ -12,6 +12,15 @@
 namespace vpic {
 
 // Grid constants passed by value to kernels (kernel-param constant bank).
+// VPIC_CHECK=1 (dev builds only: tools/check_build.sh): device-side bounds
+// checks on the hot paths' computed indices -- voxel rows gathered and
+// scattered, chunk and record slots, sort positions -- trapping on the first
+// violation (the stand-in for compute-sanitizer, closed on the GPU pool).
+#ifndef VPIC_CHECK
+#define VPIC_CHECK 0
+#endif
+#define VPIC_ASSERT(cond) do { if (VPIC_CHECK && !(cond)) __trap(); } while (0)
+
 struct GridK {
   int32_t nx, ny, nz;
   int32_t sx, sy;            // nx+2, ny+2

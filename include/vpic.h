@@ -20,11 +20,16 @@
  *      particle      vpic_particle_t, 32 B (AoS);
  *      fields[nv][8] float: ex,ey,ez,0, cbx,cby,cbz,0 (Yee: ex on the x-edge
  *                    from node (x,y,z) to (x+1,y,z), cbx on the -x face);
- *      interp[nv][24] float: ex,dexdy,dexdz,d2exdydz, ey,deydz,deydx,
- *                    d2eydzdx, ez,dezdx,dezdy,d2ezdxdy, cbx,dcbxdx,
- *                    cby,dcbydy, cbz,dcbzdz, then 6 zero pads (96 B = three
- *                    32-B sectors, so a gather is three 256-bit loads);
- *                    the array must be 32-B aligned;
+ *      interp        a buffer of nv x 24 floats holding, per voxel, the
+ *                    18 coefficients ex,dexdy,dexdz,d2exdydz, ey,deydz,
+ *                    deydx,d2eydzdx, ez,dezdx,dezdy,d2ezdxdy, cbx,dcbxdx,
+ *                    cby,dcbydy, cbz,dcbzdz, laid out as nv rows of the
+ *                    first 16 (64 B = two 32-B sectors: a gather is two
+ *                    256-bit loads) followed by nv pairs (cbz, dcbzdz)
+ *                    (8 B, four voxels per sector: one 64-bit load); the
+ *                    last nv x 24 B are unused; the array must be 32-B
+ *                    aligned (the binding's interp_coefficients() reads it
+ *                    back as [nv][18]);
  *      acc[nv][12]   float: jx[4], jy[4], jz[4] quadrant partials
  *                    (48 B = 3 x float4); jx quadrants (-y-z),(+y-z),(-y+z),(+y+z),
  *                    jy cyclic over (z,x), jz over (x,y);

@@ -164,7 +164,19 @@ k_load_interp(const GridK g, const float4 *__restrict__ f, float4 *__restrict__ 
       const int j = lane + 32 * k;
       const int src = j / 6;
       const int64_t vj = __shfl_sync(0xffffffffu, v, src);
+#if VPIC_INTERP_SPLIT
+      const int comp = j - 6 * src;
+      if (src < nact) {
+        if (comp < 4) {
+          interp[4 * vj + comp] = stage[w][j];
+        } else if (comp == 4) {   // (cbz, dcbz/dz) into the compact tail
+          const float4 q = stage[w][j];
+          reinterpret_cast<float2 *>(interp + 4 * g.nv)[vj] = make_float2(q.x, q.y);
+        }
+      }
+#else
       if (src < nact) interp[6 * vj + (j - 6 * src)] = stage[w][j];
+#endif
     }
     __syncwarp();
   }

@@ -21,6 +21,14 @@ namespace vpic {
 #endif
 #define VPIC_ASSERT(cond) do { if (VPIC_CHECK && !(cond)) __trap(); } while (0)
 
+// Interpolator layout (include/vpic.h): VPIC_INTERP_SPLIT = 1 stores the
+// first 16 coefficients of every voxel as a 64-B row (two sector-aligned
+// 32-B loads) and the last two (cbz, dcbz/dz) in a compact 8-B array after
+// the rows (4 voxels per sector), inside the same [nv][24] float buffer.
+#ifndef VPIC_INTERP_SPLIT
+#define VPIC_INTERP_SPLIT 1
+#endif
+
 struct GridK {
   int32_t nx, ny, nz;
   int32_t sx, sy;            // nx+2, ny+2

@@ -292,6 +292,18 @@ def vpic_migrate_particles_dev(ctx: Context, q: float, m: float, p, np_dev, max_
 
 
 # ------------------------------------------------------- tensor helpers --
+def interp_coefficients(interp, nv: int):
+    """The 18 interpolator coefficients per voxel, [nv][18] float32 in the
+    order of include/vpic.h, from an interp[nv][24] buffer in the library's
+    layout: nv rows of the first 16 coefficients (64 B), then nv pairs
+    (cbz, dcbz/dz) (8 B each); the last nv x 24 B are unused."""
+    import numpy as np
+    a = np.ascontiguousarray(interp.detach().cpu().numpy() if hasattr(interp, "detach") else interp,
+                             dtype=np.float32).reshape(-1)
+    rows = a[:16 * nv].reshape(nv, 16)
+    tail = a[16 * nv:18 * nv].reshape(nv, 2)
+    return np.concatenate([rows, tail], axis=1)
+
 class vpic_species_host_t(ctypes.Structure):
     _fields_ = [("q", ctypes.c_float), ("m", ctypes.c_float), ("host_in", ctypes.c_void_p),
                 ("host_out", ctypes.c_void_p), ("np", ctypes.c_int64), ("max_np", ctypes.c_int64),
